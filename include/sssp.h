@@ -1,0 +1,209 @@
+/*
+ * sssp.h -- C ABI of the B200-native ADDS single-source shortest-path library
+ * (libsssp.so, built from paper_conf_ppopp_wangfl21_b200/csrc/).
+ *
+ * Reference: K. Wang, D. Fussell, C. Lin, "A Fast Work-Efficient SSSP Algorithm
+ * for GPUs", PPoPP '21.  Citations "P:<line>" are lines of
+ * /root/reference/PAPER.md; "§8(x)" are sections of SURVEY.md.
+ *
+ * The operation (§3 "Background"): for a directed graph with
+ * non-negative edge weights and a source s, compute for every vertex v the
+ * shortest distance from s:
+ *     dist[v] = min over directed paths s ~> v of the sum of arc weights,
+ *     dist[s] = 0,   dist[v] = UINT64_MAX  iff no path exists.
+ * The method (§5) is ADDS -- asynchronous Delta-stepping with a
+ * 32-bucket approximate priority queue and a run-time Delta controller.  The
+ * schedule changes only the work performed, never the result, and all
+ * arithmetic is integer, so results are bit-exact and deterministic.
+ *
+ * Conventions
+ *  - Every entry point returns sssp_status; nothing throws across the ABI and
+ *    nothing calls exit().  On error, sssp_last_error() returns a thread-local
+ *    human-readable detail string (valid until the next call on that thread).
+ *  - Graph: CSR with n vertices and m directed arcs.  row_offsets[n+1] (uint64,
+ *    row_offsets[0]=0, non-decreasing, row_offsets[n]=m), col[m] (uint32,
+ *    < n) and w[m] (uint32 weights, any value incl. 0).  Self-loops and
+ *    parallel arcs are allowed.  n <= 2^32-2 (UINT32_MAX is a reserved id).
+ *  - Pointers passed to sssp_graph_create may be host or device memory (detected
+ *    with cudaPointerGetAttributes); the library COPIES them into its own
+ *    device memory and the caller keeps ownership.
+ *  - dist_out may be a device pointer on the graph's device (the fast path) or
+ *    host memory (the library then copies the result back before returning).
+ *  - Streams: work is enqueued on `stream` (NULL = legacy default stream).
+ *    By default a run waits for its 64-byte status block so that device-side
+ *    errors (worklist overflow, 32-bit distance overflow) can be handled
+ *    (grow the ring / switch to 64-bit distances and re-run).  With
+ *    SSSP_FLAG_ASYNC the call returns after enqueueing; the caller must
+ *    synchronise the stream and then call sssp_get_stats() to learn the status.
+ *  - Concurrency: at most one run in flight per handle (SSSP_ERR_BUSY).
+ *    Distinct handles may run concurrently on distinct streams.
+ */
+#ifndef SSSP_H_
+#define SSSP_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Same underlying type as cudaStream_t (struct CUstream_st*). */
+typedef struct CUstream_st *sssp_stream_t;
+
+typedef enum sssp_status {
+    SSSP_OK = 0,
+    SSSP_ERR_INVALID_ARGUMENT = 1, /* NULL pointer, source >= n, k == 0, bad option */
+    SSSP_ERR_INVALID_GRAPH = 2,    /* CSR validation failed; detail names the first bad index */
+    SSSP_ERR_OUT_OF_MEMORY = 3,    /* device or pinned-host allocation failed */
+    SSSP_ERR_CUDA = 4,             /* any other CUDA runtime error (detail has the CUDA string) */
+    SSSP_ERR_WORKLIST_OVERFLOW = 5,/* bucket ring full and retries exhausted / NO_RETRY set */
+    SSSP_ERR_TIMEOUT = 6,          /* device watchdog expired (options.timeout_ms) */
+    SSSP_ERR_DEVICE_MISMATCH = 7,  /* dist_out lives on another device than the graph */
+    SSSP_ERR_BUSY = 8,             /* a run is already in flight on this handle */
+    SSSP_ERR_NO_DEVICE = 9         /* no CUDA device / not an sm_100 device */
+} sssp_status;
+
+/* Options.flags bits */
+#define SSSP_FLAG_TRACE 0x1u     /* record Delta-controller samples into the trace ring (§5, Figs. 11-15 analog) */
+#define SSSP_FLAG_ASYNC 0x2u     /* do not wait for the run's status block (see Streams above) */
+#define SSSP_FLAG_NO_RETRY 0x4u  /* on worklist overflow return SSSP_ERR_WORKLIST_OVERFLOW instead of growing */
+
+/* Delta modes */
+#define SSSP_DELTA_DYNAMIC 0u    /* ADDS: run-time controller */
+#define SSSP_DELTA_STATIC 1u     /* ablation "Static-Delta": keep delta_init for the whole run */
+
+typedef struct sssp_options {
+    uint32_t struct_size;      /* = sizeof(sssp_options); set by sssp_options_default */
+    int32_t device;            /* CUDA device ordinal (default 0) */
+    uint32_t num_buckets;      /* ring size B, power of two in [2, 32]; default 32 */
+    uint32_t delta_mode;       /* SSSP_DELTA_DYNAMIC (default) or SSSP_DELTA_STATIC */
+    uint64_t delta_init;       /* initial Delta; 0 = heuristic C*W/D rounded
+                                  to the nearest power of two; else rounded to a power of two */
+    uint32_t clip_pct;         /* tail-bucket share that raises Delta and its floor; default 65 */
+    uint32_t settle_head_switches; /* K head-bucket switches between Delta changes; default 2 */
+    uint32_t util_lo_pct;      /* lower utilisation limit, % of resident threads; default 100 */
+    uint32_t util_hi_pct;      /* upper utilisation limit, % of resident threads; default 400 */
+    uint32_t dist_bits;        /* 0 = auto (32-bit internal distances when provably or observably
+                                  safe, else 64), 32 or 64 */
+    uint64_t ring_items;       /* capacity of each bucket's circular array (items, rounded up to a
+                                  power of two, >= 64); 0 = auto = max(2^16, next_pow2(n)) */
+    uint32_t flags;            /* SSSP_FLAG_* */
+    uint32_t block_threads;    /* worker CTA size: 0 = auto (256), else 128/256/512 */
+    uint32_t grid_ctas;        /* 0 = every co-resident CTA; else at most this many CTAs */
+    uint32_t batch_min;        /* minimum items a CTA claims when enough are available; 0 = auto */
+    uint32_t timeout_ms;       /* device watchdog (globaltimer); 0 = default 60000 */
+    uint32_t trace_capacity;   /* trace ring entries when SSSP_FLAG_TRACE; 0 = 65536 */
+    uint32_t active_init;      /* initial number of active (claimable) buckets; 0 = auto (1) */
+    uint32_t reserved[4];
+} sssp_options;
+
+typedef struct sssp_stats {
+    uint64_t vertices_processed; /* items expanded (not stale): the paper's work count */
+    uint64_t edges_relaxed;      /* arcs scanned from expanded items */
+    uint64_t pushes;             /* items pushed into the bucket ring (incl. the source) */
+    uint64_t stale_skips;        /* popped items whose distance was already improved */
+    uint64_t reachable;          /* vertices with finite distance  (= V_dij) */
+    uint64_t reach_edges;        /* sum of out-degrees of reachable vertices (= E_dij, GTEPS numerator) */
+    uint64_t max_dist;           /* largest finite distance */
+    uint32_t init_delta_log2;    /* log2 of the initial Delta */
+    uint32_t final_delta_log2;   /* log2 of Delta when the run ended */
+    uint32_t head_switches;      /* head-bucket advances */
+    uint32_t delta_changes;      /* Delta adjustments by the controller */
+    uint32_t retries;            /* re-runs after overflow (ring growth or 64-bit distances) */
+    uint32_t dist_bits;          /* 32 or 64: internal distance width of the last attempt */
+    uint32_t grid_ctas;          /* persistent-kernel CTAs launched */
+    uint32_t block_threads;      /* threads per CTA */
+    uint32_t runs;               /* sources covered by these stats (1 for sssp_run) */
+    uint32_t trace_entries;      /* valid entries in the trace ring (capped at capacity) */
+    float kernel_ms;             /* device time of the persistent kernel(s) (CUDA events) */
+    float total_ms;              /* device time init + kernel + finalize (CUDA events) */
+    uint32_t status;             /* sssp_status of the last run (for SSSP_FLAG_ASYNC) */
+    uint32_t reserved[3];
+} sssp_stats;
+
+/* One Delta-controller sample (written at each head-bucket switch). */
+typedef struct sssp_trace_entry {
+    uint64_t time_ns;        /* %globaltimer */
+    uint64_t head;           /* absolute head bucket number */
+    uint64_t pending_total;  /* items reserved but not completed, all buckets */
+    uint64_t pending_window; /* same, active buckets only */
+    uint64_t pending_tail;   /* same, tail (clip) bucket */
+    uint32_t delta_log2;     /* Delta in force after the switch */
+    uint32_t active;         /* active buckets after the switch */
+} sssp_trace_entry;
+
+/* Opaque handle: owns the device CSR, the workspace (bucket ring, counters,
+ * trace ring), a pinned status block and the timing events. */
+typedef struct sssp_graph sssp_graph;
+
+/* Fills *opts with the defaults documented above. NULL-safe. */
+void sssp_options_default(sssp_options *opts);
+
+/* Validates the CSR on the device (O(n+m)), copies it into library-owned
+ * device memory (interleaved {col,w} arcs), computes the graph statistics
+ * used for the initial Delta (sum of weights), and allocates the
+ * run workspace on opts->device.  opts may be NULL (defaults).
+ * Errors: INVALID_ARGUMENT (NULL out or arrays / n == 0 / n > 2^32-2),
+ * INVALID_GRAPH (detail names the first offending index), OUT_OF_MEMORY,
+ * NO_DEVICE, CUDA.  On error *out is set to NULL and nothing leaks. */
+sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t *row_offsets,
+                              const uint32_t *col, const uint32_t *w,
+                              const sssp_options *opts, sssp_graph **out);
+
+/* Releases everything the handle owns (synchronises its device first). NULL-safe. */
+sssp_status sssp_graph_destroy(sssp_graph *g);
+
+/* Replaces the run-time options of an existing handle (Delta mode/initial
+ * Delta, controller constants, ring size, grid/block shape, flags).  The
+ * device, and the CSR, cannot change.  Not allowed while a run is in flight. */
+sssp_status sssp_set_options(sssp_graph *g, const sssp_options *opts);
+
+/* Single-source run: dist_out[v] (uint64, n entries) = exact distance from
+ * `source`, UINT64_MAX when unreachable.  Enqueued on `stream`; see
+ * "Streams" for the synchronous default and SSSP_FLAG_ASYNC.
+ * Errors: INVALID_ARGUMENT (source >= n, NULL dist_out), DEVICE_MISMATCH,
+ * BUSY, WORKLIST_OVERFLOW (only with NO_RETRY or after 4 growths), TIMEOUT,
+ * CUDA. */
+sssp_status sssp_run(sssp_graph *g, uint32_t source, uint64_t *dist_out, sssp_stream_t stream);
+
+/* Multi-source batch: k sources (host array), results row-major
+ * dist_out[i*n + v] for source i (k*n uint64 entries, device or host).
+ * Equivalent to k calls of sssp_run (bit-identical), amortising launch and
+ * status overheads; stats cover the whole batch.  Errors as sssp_run plus
+ * INVALID_ARGUMENT for k == 0 or any source >= n (checked before any work). */
+sssp_status sssp_run_batch(sssp_graph *g, const uint32_t *sources, uint32_t k,
+                           uint64_t *dist_out, sssp_stream_t stream);
+
+/* Statistics of the last run/batch (valid after the run's stream is
+ * synchronised).  With SSSP_FLAG_ASYNC this also performs the deferred
+ * status check and returns the run's status. */
+sssp_status sssp_get_stats(sssp_graph *g, sssp_stats *out);
+
+/* Copies up to `cap` trace entries of the last run (SSSP_FLAG_TRACE) into
+ * host memory `out`; *count receives the number copied. */
+sssp_status sssp_get_trace(sssp_graph *g, sssp_trace_entry *out, uint32_t cap, uint32_t *count);
+
+/* Graph facts: n, m, sum of weights, max weight, and the heuristic initial
+ * Delta (log2) = round(log2(C * W / D)), C = 32, W = sum_w/m, D = m/n. */
+sssp_status sssp_graph_info(const sssp_graph *g, uint32_t *n, uint64_t *m, uint64_t *sum_w,
+                            uint32_t *max_w, uint32_t *heuristic_delta_log2);
+
+/* The bucket ring's priority mapping (§5.4-5.5), exposed for unit
+ * tests: the ring offset (0 = head ... B-1 = tail) that an item of distance d
+ * is pushed to when the head bucket is number `head` (absolute, in units of
+ * Delta = 2^delta_log2) and the ring has B buckets: floor(d / Delta) - head,
+ * clamped to [0, B-1] (items beyond the ring are clipped into the tail,
+ * P:195).  Pure function, no device needed. */
+uint32_t sssp_bucket_offset(uint64_t d, uint32_t delta_log2, uint64_t head, uint32_t num_buckets);
+
+/* Static description strings. */
+const char *sssp_status_string(sssp_status st);
+const char *sssp_last_error(void);
+/* Library build string (arch, version). */
+const char *sssp_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SSSP_H_ */

@@ -1,0 +1,256 @@
+"""B200-native ADDS single-source shortest paths (PPoPP'21 hot path).
+
+Thin ctypes binding over ``libsssp.so`` (``include/sssp.h``): argument
+marshalling only -- every step of the SSSP runs in the sm_100a kernels under
+``csrc/``.  There is no CPU fallback: if the extension is not built, or no
+sm_100 device is present, calls raise.
+
+PyTorch is used for device memory (output tensors) and streams only.
+
+    >>> import paper_conf_ppopp_wangfl21_b200 as sssp
+    >>> g = sssp.Graph(row_offsets, col, w)          # numpy / torch (host or cuda)
+    >>> d = g.run(source)                            # torch.int64 [n] on cuda (UINT64_MAX -> -1)
+    >>> D = g.run_batch(sources)                     # torch.int64 [k, n]
+    >>> g.stats()                                    # dict (work counts, Delta, timings)
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+from . import _build
+
+LIB_PATH = _build.LIB
+_lib = None
+
+INF = 0xFFFFFFFFFFFFFFFF
+
+SSSP_FLAG_TRACE = 0x1
+SSSP_FLAG_ASYNC = 0x2
+SSSP_FLAG_NO_RETRY = 0x4
+SSSP_DELTA_DYNAMIC = 0
+SSSP_DELTA_STATIC = 1
+
+STATUS = {
+    0: "SSSP_OK", 1: "SSSP_ERR_INVALID_ARGUMENT", 2: "SSSP_ERR_INVALID_GRAPH", 3: "SSSP_ERR_OUT_OF_MEMORY",
+    4: "SSSP_ERR_CUDA", 5: "SSSP_ERR_WORKLIST_OVERFLOW", 6: "SSSP_ERR_TIMEOUT", 7: "SSSP_ERR_DEVICE_MISMATCH",
+    8: "SSSP_ERR_BUSY", 9: "SSSP_ERR_NO_DEVICE",
+}
+
+
+class SSSPError(RuntimeError):
+    def __init__(self, status: int, detail: str):
+        super().__init__(f"{STATUS.get(status, status)}: {detail}")
+        self.status = status
+        self.detail = detail
+
+
+class sssp_options(ctypes.Structure):
+    _fields_ = [
+        ("struct_size", ctypes.c_uint32), ("device", ctypes.c_int32), ("num_buckets", ctypes.c_uint32),
+        ("delta_mode", ctypes.c_uint32), ("delta_init", ctypes.c_uint64), ("clip_pct", ctypes.c_uint32),
+        ("settle_head_switches", ctypes.c_uint32), ("util_lo_pct", ctypes.c_uint32),
+        ("util_hi_pct", ctypes.c_uint32), ("dist_bits", ctypes.c_uint32), ("ring_items", ctypes.c_uint64),
+        ("flags", ctypes.c_uint32), ("block_threads", ctypes.c_uint32), ("grid_ctas", ctypes.c_uint32),
+        ("batch_min", ctypes.c_uint32), ("timeout_ms", ctypes.c_uint32), ("trace_capacity", ctypes.c_uint32),
+        ("active_init", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 4),
+    ]
+
+
+class sssp_stats(ctypes.Structure):
+    _fields_ = [
+        ("vertices_processed", ctypes.c_uint64), ("edges_relaxed", ctypes.c_uint64), ("pushes", ctypes.c_uint64),
+        ("stale_skips", ctypes.c_uint64), ("reachable", ctypes.c_uint64), ("reach_edges", ctypes.c_uint64),
+        ("max_dist", ctypes.c_uint64), ("init_delta_log2", ctypes.c_uint32), ("final_delta_log2", ctypes.c_uint32),
+        ("head_switches", ctypes.c_uint32), ("delta_changes", ctypes.c_uint32), ("retries", ctypes.c_uint32),
+        ("dist_bits", ctypes.c_uint32), ("grid_ctas", ctypes.c_uint32), ("block_threads", ctypes.c_uint32),
+        ("runs", ctypes.c_uint32), ("trace_entries", ctypes.c_uint32), ("kernel_ms", ctypes.c_float),
+        ("total_ms", ctypes.c_float), ("status", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3),
+    ]
+
+
+class sssp_trace_entry(ctypes.Structure):
+    _fields_ = [
+        ("time_ns", ctypes.c_uint64), ("head", ctypes.c_uint64), ("pending_total", ctypes.c_uint64),
+        ("pending_window", ctypes.c_uint64), ("pending_tail", ctypes.c_uint64), ("delta_log2", ctypes.c_uint32),
+        ("active", ctypes.c_uint32),
+    ]
+
+
+# (name, restype, argtypes) for every symbol declared in include/sssp.h
+_P = ctypes.c_void_p
+SIGNATURES = [
+    ("sssp_options_default", None, [ctypes.POINTER(sssp_options)]),
+    ("sssp_graph_create", ctypes.c_int,
+     [ctypes.c_uint32, ctypes.c_uint64, _P, _P, _P, ctypes.POINTER(sssp_options), ctypes.POINTER(_P)]),
+    ("sssp_graph_destroy", ctypes.c_int, [_P]),
+    ("sssp_set_options", ctypes.c_int, [_P, ctypes.POINTER(sssp_options)]),
+    ("sssp_run", ctypes.c_int, [_P, ctypes.c_uint32, _P, _P]),
+    ("sssp_run_batch", ctypes.c_int, [_P, _P, ctypes.c_uint32, _P, _P]),
+    ("sssp_get_stats", ctypes.c_int, [_P, ctypes.POINTER(sssp_stats)]),
+    ("sssp_get_trace", ctypes.c_int, [_P, _P, ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint32)]),
+    ("sssp_graph_info", ctypes.c_int, [_P, _P, _P, _P, _P, _P]),
+    ("sssp_bucket_offset", ctypes.c_uint32, [ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_uint32]),
+    ("sssp_status_string", ctypes.c_char_p, [ctypes.c_int]),
+    ("sssp_last_error", ctypes.c_char_p, []),
+    ("sssp_version", ctypes.c_char_p, []),
+]
+
+
+def lib():
+    """Load libsssp.so (raises if it was not built: there is no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is missing: build the CUDA extension first "
+                               "(python -c 'import __graft_entry__ as g; g.build()')")
+        L = ctypes.CDLL(LIB_PATH)
+        for name, res, args in SIGNATURES:
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def _check(st: int):
+    if st != 0:
+        raise SSSPError(st, lib().sssp_last_error().decode())
+
+
+# ------------------------------------------------------------------ same-name C wrappers
+def sssp_options_default(**overrides) -> sssp_options:
+    o = sssp_options()
+    lib().sssp_options_default(ctypes.byref(o))
+    for k, v in overrides.items():
+        if not hasattr(o, k):
+            raise KeyError(k)
+        setattr(o, k, v)
+    return o
+
+
+def sssp_bucket_offset(d: int, delta_log2: int, head: int, num_buckets: int = 32) -> int:
+    return int(lib().sssp_bucket_offset(d, delta_log2, head, num_buckets))
+
+
+def sssp_status_string(st: int) -> str:
+    return lib().sssp_status_string(st).decode()
+
+
+def sssp_version() -> str:
+    return lib().sssp_version().decode()
+
+
+def _as_host_or_dev(a, dtype):
+    """Return (pointer, keepalive) for a numpy array or a torch tensor (host or cuda)."""
+    try:
+        import torch
+        if isinstance(a, torch.Tensor):
+            t = a.contiguous()
+            return t.data_ptr(), t
+    except ImportError:  # pragma: no cover
+        pass
+    arr = np.ascontiguousarray(a, dtype=dtype)
+    return arr.ctypes.data, arr
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+class Graph:
+    """A CSR graph resident on one GPU plus its ADDS workspace (``sssp_graph*``)."""
+
+    def __init__(self, row_offsets, col, w, options: sssp_options | None = None, device: int = 0, **opt):
+        L = lib()
+        self._h = _P()
+        if options is None:
+            options = sssp_options_default(device=device, **opt)
+        self.options = options
+        self.n = int(len(row_offsets) - 1)
+        self.m = int(len(col))
+        po, k1 = _as_host_or_dev(row_offsets, np.uint64)
+        pc, k2 = _as_host_or_dev(col, np.uint32)
+        pw, k3 = _as_host_or_dev(w, np.uint32)
+        _check(L.sssp_graph_create(self.n, self.m, po, pc, pw, ctypes.byref(options), ctypes.byref(self._h)))
+        self.device = options.device
+
+    @classmethod
+    def from_csr(cls, csr, **kw):
+        return cls(csr.row_offsets, csr.col, csr.w, **kw)
+
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            lib().sssp_graph_destroy(self._h)
+            self._h = _P()
+
+    __del__ = close
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def set_options(self, **overrides):
+        o = sssp_options()
+        ctypes.memmove(ctypes.byref(o), ctypes.byref(self.options), ctypes.sizeof(o))
+        for k, v in overrides.items():
+            setattr(o, k, v)
+        _check(lib().sssp_set_options(self._h, ctypes.byref(o)))
+        self.options = o
+
+    def run(self, source: int, out=None, stream=None):
+        """dist[v] from ``source`` as a torch.int64 cuda tensor (UINT64_MAX reads as -1)."""
+        import torch
+        if out is None:
+            out = torch.empty(self.n, dtype=torch.int64, device=f"cuda:{self.device}")
+        _check(lib().sssp_run(self._h, int(source), out.data_ptr(), _stream_ptr(stream)))
+        return out
+
+    def run_host(self, source: int, out: np.ndarray | None = None, stream=None) -> np.ndarray:
+        """Same, into host memory (the library copies the result back)."""
+        if out is None:
+            out = np.empty(self.n, dtype=np.uint64)
+        _check(lib().sssp_run(self._h, int(source), out.ctypes.data, _stream_ptr(stream)))
+        return out
+
+    def run_batch(self, sources, out=None, stream=None):
+        """[k, n] torch.int64 distances for k sources (row i <-> sources[i])."""
+        import torch
+        src = np.ascontiguousarray(sources, dtype=np.uint32)
+        if out is None:
+            out = torch.empty((len(src), self.n), dtype=torch.int64, device=f"cuda:{self.device}")
+        _check(lib().sssp_run_batch(self._h, src.ctypes.data, len(src), out.data_ptr(), _stream_ptr(stream)))
+        return out
+
+    def stats(self) -> dict:
+        s = sssp_stats()
+        _check(lib().sssp_get_stats(self._h, ctypes.byref(s)))
+        d = {f: getattr(s, f) for f, _ in sssp_stats._fields_ if f != "reserved"}
+        return d
+
+    def trace(self):
+        cap = self.options.trace_capacity or 65536
+        buf = (sssp_trace_entry * cap)()
+        cnt = ctypes.c_uint32(0)
+        _check(lib().sssp_get_trace(self._h, buf, cap, ctypes.byref(cnt)))
+        return [{f: getattr(buf[i], f) for f, _ in sssp_trace_entry._fields_} for i in range(cnt.value)]
+
+    def info(self) -> dict:
+        n, m, sw, mw, hk = ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_uint32(), ctypes.c_uint32()
+        _check(lib().sssp_graph_info(self._h, ctypes.byref(n), ctypes.byref(m), ctypes.byref(sw), ctypes.byref(mw),
+                                     ctypes.byref(hk)))
+        return {"n": n.value, "m": m.value, "sum_w": sw.value, "max_w": mw.value, "heuristic_delta_log2": hk.value}
+
+
+def to_u64(t) -> np.ndarray:
+    """torch.int64 distances -> numpy uint64 (UINT64_MAX for unreachable)."""
+    return t.detach().cpu().numpy().view(np.uint64)

@@ -1,0 +1,106 @@
+// aux_kernels.cuh -- create-time and per-run helper kernels (grid-stride, sm_100a).
+//   validate_csr   O(n+m) CSR checks (§8(b) "Validation at create")
+//   interleave     {col, w} -> 8-byte arcs + sum/max of weights (initial Delta)
+//   init_run       dist = inf, dist[s] = 0, ring counters reset, source item pushed (§8(a) A3)
+//   finalize       widen dist to uint64 (inf -> UINT64_MAX) + reach / E_dij / max (§8(a) A10)
+#pragma once
+#include "common.cuh"
+
+namespace adds {
+
+__global__ void validate_csr_kernel(const unsigned long long* __restrict__ off, const unsigned* __restrict__ col,
+                                    unsigned n, unsigned long long m, unsigned long long* bad) {
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+        if (off[v] > off[v + 1]) atomicMin(&bad[0], v);
+    for (unsigned long long e = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; e < m; e += stride)
+        if (col[e] >= n) atomicMin(&bad[1], e);
+}
+
+__global__ void interleave_kernel(const unsigned* __restrict__ col, const unsigned* __restrict__ w,
+                                  uint2* __restrict__ adj, unsigned long long m, unsigned long long* sum_w,
+                                  unsigned* max_w) {
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    unsigned long long s = 0;
+    unsigned mx = 0;
+    for (unsigned long long e = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; e < m; e += stride) {
+        const unsigned ww = w[e];
+        adj[e] = make_uint2(col[e], ww);
+        s += ww;
+        mx = ww > mx ? ww : mx;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        s += __shfl_xor_sync(0xffffffffu, s, o);
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    }
+    if ((threadIdx.x & 31) == 0) {
+        atomicAdd(sum_w, s);
+        atomicMax(max_w, mx);
+    }
+}
+
+template <typename DistT>
+__global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned source, Ctl* ctl, BucketCtl* bk,
+                                char* ring, unsigned long long cap, Head h0) {
+    using IT = ItemT<DistT>;
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+        dist[v] = (v == source) ? (DistT)0 : DistInf<DistT>::value;
+    if (blockIdx.x == 0) {
+        const unsigned t = threadIdx.x;
+        if (t < kMaxBuckets) {
+            bk[t].reserve.v = 0;
+            bk[t].avail.v = 0;
+            bk[t].claim.v = 0;
+            bk[t].done.v = 0;
+            if (t == meta_hs(h0.meta)) {  // the source item: bucket 0 = head ("initially ... infinity")
+                IT::store(ring + (size_t)t * cap * IT::kBytes, IT::make(source, 0ull));
+                bk[t].reserve.v = 1;
+                bk[t].avail.v = 1;
+            }
+        }
+        if (t == 0) {
+            ctl->head = h0;
+            ctl->outstanding = 1;
+            ctl->status = 0;
+            ctl->trace_count = 0;
+            ctl->head_switches = 0;
+            ctl->delta_changes = 0;
+            ctl->t_start = globaltimer();
+            ctl->st_vertices = ctl->st_edges = ctl->st_pushes = ctl->st_stale = 0;
+            ctl->reach_v = ctl->reach_e = ctl->max_dist = 0;
+        }
+    }
+}
+
+template <typename DistT>
+__global__ void finalize_kernel(const DistT* __restrict__ dist, unsigned long long* __restrict__ out, unsigned n,
+                                const unsigned long long* __restrict__ off, Ctl* ctl) {
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    unsigned long long rv = 0, re = 0, mx = 0;
+    for (unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
+        const DistT d = dist[v];
+        if (d == DistInf<DistT>::value) {
+            out[v] = ~0ull;
+        } else {
+            out[v] = (unsigned long long)d;
+            rv += 1;
+            re += off[v + 1] - off[v];
+            mx = (unsigned long long)d > mx ? (unsigned long long)d : mx;
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        rv += __shfl_xor_sync(0xffffffffu, rv, o);
+        re += __shfl_xor_sync(0xffffffffu, re, o);
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    }
+    if ((threadIdx.x & 31) == 0 && rv) {
+        atomicAdd(&ctl->reach_v, rv);
+        atomicAdd(&ctl->reach_e, re);
+        atomicMax(&ctl->max_dist, mx);
+    }
+}
+
+}  // namespace adds

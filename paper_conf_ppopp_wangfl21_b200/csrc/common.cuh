@@ -1,0 +1,216 @@
+// common.cuh -- device data structures and PTX helpers of the ADDS worklist.
+//
+// Layout in HBM:
+//   BucketCtl[32]  per ring slot: reserve (P:159 resv_ptr), avail (published -
+//                  claimed gate), claim (P:159 read_ptr), done (P:176 CWC);
+//                  every counter on its own 128-B line so the L2 atomic units
+//                  of different counters never serialise on one line.
+//   Ctl            head state (16 B, 128-bit CAS), outstanding-work counter
+//                  (termination), status bits, statistics, trace cursor.
+//   ring           nb circular arrays of C items each (pre-allocated).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace adds {
+
+constexpr uint32_t kMaxBuckets = 32;
+
+// status bits written by the device
+constexpr unsigned kStRingOverflow = 1u;   // a bucket's circular array would lap an unclaimed item
+constexpr unsigned kStDistOverflow = 2u;   // 32-bit distance would overflow -> rerun with 64-bit
+constexpr unsigned kStTimeout = 4u;        // watchdog
+constexpr unsigned kStBug = 8u;            // internal invariant violated
+
+struct alignas(128) Counter {
+    unsigned long long v;
+    unsigned long long pad_[15];
+};
+
+struct BucketCtl {
+    Counter reserve;  // items reserved by writers (monotone)      = resv_ptr
+    Counter avail;    // signed: published and not yet claimed      (claim gate)
+    Counter claim;    // items claimed by workers (monotone)        = read_ptr
+    Counter done;     // items whose processing completed           = CWC
+};
+
+// Head state, updated only by 128-bit CAS (one writer per head switch).
+//   h    : absolute number of the head bucket (units of Delta = 2^k)
+//   meta : [0,8) hs = ring slot of the head  [8,16) k = log2 Delta
+//          [16,24) A = active buckets        [24,32) floor of k (clip bound)
+//          [32,48) head switches since the last Delta change
+struct alignas(16) Head {
+    unsigned long long h;
+    unsigned long long meta;
+};
+
+__host__ __device__ __forceinline__ unsigned long long pack_meta(unsigned hs, unsigned k, unsigned A,
+                                                                 unsigned flo, unsigned since) {
+    return (unsigned long long)(hs & 0xff) | ((unsigned long long)(k & 0xff) << 8) |
+           ((unsigned long long)(A & 0xff) << 16) | ((unsigned long long)(flo & 0xff) << 24) |
+           ((unsigned long long)(since & 0xffff) << 32);
+}
+__host__ __device__ __forceinline__ unsigned meta_hs(unsigned long long m) { return (unsigned)(m & 0xff); }
+__host__ __device__ __forceinline__ unsigned meta_k(unsigned long long m) { return (unsigned)((m >> 8) & 0xff); }
+__host__ __device__ __forceinline__ unsigned meta_A(unsigned long long m) { return (unsigned)((m >> 16) & 0xff); }
+__host__ __device__ __forceinline__ unsigned meta_floor(unsigned long long m) { return (unsigned)((m >> 24) & 0xff); }
+__host__ __device__ __forceinline__ unsigned meta_since(unsigned long long m) { return (unsigned)((m >> 32) & 0xffff); }
+
+struct TraceEntry {  // mirrors sssp_trace_entry
+    unsigned long long time_ns, head, pending_total, pending_window, pending_tail;
+    unsigned delta_log2, active;
+};
+
+struct alignas(128) Ctl {
+    Head head;
+    char pad0_[128 - sizeof(Head)];
+    long long outstanding;  // pushed - completed; 0 <=> quiescent (termination, P:182 reading R11)
+    char pad1_[120];
+    unsigned status;
+    unsigned trace_count;
+    unsigned head_switches;
+    unsigned delta_changes;
+    unsigned long long t_start;  // %globaltimer at init (watchdog)
+    char pad2_[104];
+    // statistics (flushed once per CTA at exit, or by finalize)
+    unsigned long long st_vertices, st_edges, st_pushes, st_stale;
+    unsigned long long reach_v, reach_e, max_dist;
+    unsigned long long pad3_[9];
+};
+static_assert(sizeof(Ctl) % 128 == 0, "Ctl layout");
+
+// ------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ long long ld_relaxed_s64(const long long* p) {
+    long long v;
+    asm volatile("ld.relaxed.gpu.global.s64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned ld_relaxed_u32(const unsigned* p) {
+    unsigned v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void ld_relaxed_v2u64(const void* p, unsigned long long& a, unsigned long long& b) {
+    asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_u64(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_v2u64(void* p, unsigned long long a, unsigned long long b) {
+    asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
+}
+// dist loads go to L2 (.cg): dist is updated by L2 atomics, an L1-stale value is
+// still a valid upper bound (it only weakens the filter) but L2 is fresher.
+__device__ __forceinline__ unsigned ld_cg(const unsigned* p) { return __ldcg(p); }
+__device__ __forceinline__ unsigned long long ld_cg(const unsigned long long* p) { return __ldcg(p); }
+
+__device__ __forceinline__ unsigned long long globaltimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+// 128-bit CAS on the head state (sm_90+: atom.cas.b128).
+__device__ __forceinline__ bool cas_head(Head* addr, Head expect, Head desired, Head& seen) {
+    unsigned long long o0, o1;
+    asm volatile(
+        "{\n\t.reg .b128 d, b, c;\n\t"
+        "mov.b128 b, {%2, %3};\n\t"
+        "mov.b128 c, {%4, %5};\n\t"
+        "atom.relaxed.gpu.global.cas.b128 d, [%6], b, c;\n\t"
+        "mov.b128 {%0, %1}, d;\n\t}"
+        : "=l"(o0), "=l"(o1)
+        : "l"(expect.h), "l"(expect.meta), "l"(desired.h), "l"(desired.meta), "l"(addr)
+        : "memory");
+    seen.h = o0;
+    seen.meta = o1;
+    return o0 == expect.h && o1 == expect.meta;
+}
+
+__device__ __forceinline__ Head ld_head(const Head* p) {
+    Head h;
+    ld_relaxed_v2u64(p, h.h, h.meta);
+    return h;
+}
+
+__device__ __forceinline__ unsigned lanemask_lt() {
+    unsigned m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+// ------------------------------------------------------------ item formats
+// 32-bit distances: one 64-bit word  (v | d << 32); empty = all ones (v = 2^32-1
+// is a reserved id).  A single 64-bit store is single-copy atomic, so writing
+// the item IS its publication: no write-completed counter and no fence per item
+// (D2, replaces P:161's WCC).
+// 64-bit distances: 16 bytes {v, d}; empty = both all ones; valid once both
+// words are written (each 8-byte element is single-copy atomic).
+template <typename DistT>
+struct ItemT;
+
+template <>
+struct ItemT<uint32_t> {
+    using Raw = unsigned long long;
+    static constexpr int kBytes = 8;
+    __device__ __forceinline__ static Raw make(uint32_t v, unsigned long long d) {
+        return (unsigned long long)v | (d << 32);
+    }
+    __device__ __forceinline__ static bool load(const void* slot, uint32_t& v, unsigned long long& d) {
+        unsigned long long x = ld_relaxed_u64((const unsigned long long*)slot);
+        v = (uint32_t)x;
+        d = x >> 32;
+        return x != ~0ull;
+    }
+    __device__ __forceinline__ static bool empty(const void* slot) {
+        return ld_relaxed_u64((const unsigned long long*)slot) == ~0ull;
+    }
+    __device__ __forceinline__ static void store(void* slot, Raw r) { st_relaxed_u64((unsigned long long*)slot, r); }
+    __device__ __forceinline__ static void clear(void* slot) { st_relaxed_u64((unsigned long long*)slot, ~0ull); }
+};
+
+template <>
+struct ItemT<unsigned long long> {
+    struct Raw {
+        unsigned long long v, d;
+    };
+    static constexpr int kBytes = 16;
+    __device__ __forceinline__ static Raw make(uint32_t v, unsigned long long d) { return Raw{v, d}; }
+    __device__ __forceinline__ static bool load(const void* slot, uint32_t& v, unsigned long long& d) {
+        unsigned long long a, b;
+        ld_relaxed_v2u64(slot, a, b);
+        v = (uint32_t)a;
+        d = b;
+        return a != ~0ull && b != ~0ull;
+    }
+    __device__ __forceinline__ static bool empty(const void* slot) {
+        unsigned long long a, b;
+        ld_relaxed_v2u64(slot, a, b);
+        return a == ~0ull && b == ~0ull;
+    }
+    __device__ __forceinline__ static void store(void* slot, Raw r) { st_relaxed_v2u64(slot, r.v, r.d); }
+    __device__ __forceinline__ static void clear(void* slot) { st_relaxed_v2u64(slot, ~0ull, ~0ull); }
+};
+
+template <typename DistT>
+struct DistInf;
+template <>
+struct DistInf<uint32_t> {
+    static constexpr uint32_t value = 0xFFFFFFFFu;
+};
+template <>
+struct DistInf<unsigned long long> {
+    static constexpr unsigned long long value = ~0ull;
+};
+
+}  // namespace adds

@@ -1,0 +1,630 @@
+// sssp_lib.cu -- the C ABI of include/sssp.h: handle, validation, options,
+// workspace, launch sequence, status handling and retry.  All compute runs in
+// the kernels of adds_kernel.cuh / aux_kernels.cuh; there is no CPU fallback.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "../../include/sssp.h"
+#include "adds_kernel.cuh"
+#include "aux_kernels.cuh"
+#include "bucket_map.h"
+
+using namespace adds;
+
+static_assert(sizeof(TraceEntry) == sizeof(sssp_trace_entry), "trace layout");
+
+namespace {
+
+thread_local std::string g_err;
+
+sssp_status fail(sssp_status st, const std::string& msg) {
+    g_err = msg;
+    return st;
+}
+
+sssp_status cuda_fail(cudaError_t e, const char* what) {
+    cudaGetLastError();  // clear sticky-free errors
+    if (e == cudaErrorMemoryAllocation) return fail(SSSP_ERR_OUT_OF_MEMORY, std::string(what) + ": out of device memory");
+    return fail(SSSP_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+#define CK(call, what)                                   \
+    do {                                                 \
+        cudaError_t e_ = (call);                         \
+        if (e_ != cudaSuccess) return cuda_fail(e_, what); \
+    } while (0)
+
+unsigned long long next_pow2(unsigned long long x) {
+    unsigned long long p = 1;
+    while (p < x) p <<= 1;
+    return p;
+}
+unsigned ilog2_round(double x) {
+    if (!(x > 1.0)) return 0;
+    double l = std::log2(x);
+    long r = std::lround(l);
+    return r < 0 ? 0u : (unsigned)r;
+}
+
+struct DevBuf {
+    void* p = nullptr;
+    size_t bytes = 0;
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        bytes = 0;
+    }
+};
+
+}  // namespace
+
+struct sssp_graph {
+    int device = 0;
+    uint32_t n = 0;
+    uint64_t m = 0;
+    unsigned long long* d_off = nullptr;
+    uint2* d_adj = nullptr;
+    uint64_t sum_w = 0;
+    uint32_t max_w = 0;
+    uint32_t heur_k = 0;
+    sssp_options opts{};
+    int sm_count = 0;
+
+    DevBuf dist;        // 8n bytes (serves 32- and 64-bit distances)
+    DevBuf ring;        // nb * cap * item bytes
+    unsigned long long cap = 0;
+    int ring_item_bytes = 0;
+    DevBuf bk, ctl, trace, scratch, hostout;
+    unsigned trace_alloc = 0;
+    Ctl* h_ctl = nullptr;  // pinned
+    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+
+    int cur_bits = 32;  // 64 after a 32-bit overflow was observed (sticky)
+    bool busy = false;
+    bool async_pending = false;
+    sssp_stats stats{};
+    uint32_t last_grid = 0, last_block = 0, last_k0 = 0;
+};
+
+namespace {
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+sssp_status check_options(const sssp_options& o) {
+    if (o.struct_size != sizeof(sssp_options)) return fail(SSSP_ERR_INVALID_ARGUMENT, "options.struct_size mismatch");
+    if (o.num_buckets < 2 || o.num_buckets > 32 || (o.num_buckets & (o.num_buckets - 1)))
+        return fail(SSSP_ERR_INVALID_ARGUMENT, "num_buckets must be a power of two in [2, 32]");
+    if (o.delta_mode > 1) return fail(SSSP_ERR_INVALID_ARGUMENT, "delta_mode");
+    if (o.dist_bits != 0 && o.dist_bits != 32 && o.dist_bits != 64) return fail(SSSP_ERR_INVALID_ARGUMENT, "dist_bits");
+    if (o.block_threads != 0 && o.block_threads != 128 && o.block_threads != 256 && o.block_threads != 512)
+        return fail(SSSP_ERR_INVALID_ARGUMENT, "block_threads must be 0, 128, 256 or 512");
+    if (o.clip_pct == 0 || o.clip_pct > 100) return fail(SSSP_ERR_INVALID_ARGUMENT, "clip_pct");
+    if (o.active_init > o.num_buckets) return fail(SSSP_ERR_INVALID_ARGUMENT, "active_init > num_buckets");
+    return SSSP_OK;
+}
+
+// ----------------------------------------------------------------- kernel table
+template <typename DistT, int BT>
+void* kfun() {
+    return (void*)adds_persistent_kernel<DistT, BT>;
+}
+void* persistent_fn(int bits, int bt) {
+    if (bits == 32) {
+        if (bt == 128) return kfun<uint32_t, 128>();
+        if (bt == 512) return kfun<uint32_t, 512>();
+        return kfun<uint32_t, 256>();
+    }
+    if (bt == 128) return kfun<unsigned long long, 128>();
+    if (bt == 512) return kfun<unsigned long long, 512>();
+    return kfun<unsigned long long, 256>();
+}
+
+sssp_status ensure_ring(sssp_graph* g, int item_bytes, unsigned long long cap) {
+    const size_t bytes = (size_t)g->opts.num_buckets * cap * item_bytes;
+    if (g->ring.p && g->ring.bytes >= bytes && g->cap == cap && g->ring_item_bytes == item_bytes) return SSSP_OK;
+    g->ring.release();
+    CK(cudaMalloc(&g->ring.p, bytes), "allocating the bucket ring");
+    g->ring.bytes = bytes;
+    CK(cudaMemset(g->ring.p, 0xFF, bytes), "clearing the bucket ring");
+    g->cap = cap;
+    g->ring_item_bytes = item_bytes;
+    return SSSP_OK;
+}
+
+sssp_status ensure_trace(sssp_graph* g) {
+    if (!(g->opts.flags & SSSP_FLAG_TRACE)) return SSSP_OK;
+    unsigned cap = g->opts.trace_capacity ? g->opts.trace_capacity : 65536u;
+    if (g->trace.p && g->trace_alloc >= cap) return SSSP_OK;
+    g->trace.release();
+    CK(cudaMalloc(&g->trace.p, (size_t)cap * sizeof(TraceEntry)), "allocating the trace ring");
+    g->trace_alloc = cap;
+    return SSSP_OK;
+}
+
+unsigned long long default_cap(const sssp_graph* g) {
+    if (g->opts.ring_items) return next_pow2(std::max<unsigned long long>(g->opts.ring_items, 64ull));
+    return next_pow2(std::max<unsigned long long>((unsigned long long)g->n, 1ull << 16));
+}
+
+template <typename DistT>
+Params<DistT> make_params(sssp_graph* g, unsigned grid, unsigned bt, unsigned k_max) {
+    Params<DistT> p{};
+    p.off = g->d_off;
+    p.adj = g->d_adj;
+    p.dist = (DistT*)g->dist.p;
+    p.ring = (char*)g->ring.p;
+    p.bk = (BucketCtl*)g->bk.p;
+    p.ctl = (Ctl*)g->ctl.p;
+    const bool tr = (g->opts.flags & SSSP_FLAG_TRACE) != 0;
+    p.trace = tr ? (TraceEntry*)g->trace.p : nullptr;
+    p.trace_cap = tr ? g->trace_alloc : 0;
+    p.n = g->n;
+    p.nb = g->opts.num_buckets;
+    p.cap = g->cap;
+    p.dynamic = g->opts.delta_mode == SSSP_DELTA_DYNAMIC;
+    p.clip_pct = g->opts.clip_pct;
+    p.settle = g->opts.settle_head_switches;
+    p.util_lo_pct = g->opts.util_lo_pct;
+    p.util_hi_pct = g->opts.util_hi_pct;
+    p.resident_threads = (unsigned long long)grid * bt;
+    const double deg = g->n ? (double)g->m / g->n : 0.0;
+    p.avg_deg_x16 = (unsigned)std::min(16.0 * deg + 0.5, 4.0e9);
+    p.batch_min = g->opts.batch_min ? g->opts.batch_min : 32;
+    unsigned sh = 0;
+    while ((1u << (sh + 1)) <= grid) ++sh;  // floor(log2 grid)
+    p.share_shift = sh > 2 ? sh - 2 : 0;
+    p.k_max = k_max;
+    p.timeout_ns = (unsigned long long)(g->opts.timeout_ms ? g->opts.timeout_ms : 60000u) * 1000000ull;
+    return p;
+}
+
+// One attempt of one source with `bits`-wide internal distances.
+template <typename DistT>
+sssp_status launch_one(sssp_graph* g, uint32_t source, unsigned long long* out_dev, cudaStream_t s, int bits,
+                       unsigned k0) {
+    const unsigned bt = g->opts.block_threads ? g->opts.block_threads : 256;
+    void* fn = persistent_fn(bits, (int)bt);
+    int occ = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, (int)bt, 0), "occupancy query");
+    if (occ < 1) return fail(SSSP_ERR_CUDA, "persistent kernel cannot be resident");
+    unsigned grid = (unsigned)(occ * g->sm_count);
+    if (g->opts.grid_ctas && g->opts.grid_ctas < grid) grid = g->opts.grid_ctas;
+    const unsigned k_max = bits == 32 ? 31u : 63u;
+    unsigned k = std::min(k0, k_max);
+    const unsigned A0 = g->opts.active_init ? g->opts.active_init : 1u;
+    Head h0{0ull, pack_meta(0, k, A0, 0, 0)};
+    Params<DistT> p = make_params<DistT>(g, grid, bt, k_max);
+
+    const unsigned aux_grid = (unsigned)g->sm_count * 8;
+    CK(cudaEventRecord(g->ev[0], s), "event");
+    init_run_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, g->n, source, p.ctl, p.bk, p.ring, g->cap, h0);
+    CK(cudaGetLastError(), "init kernel launch");
+    CK(cudaEventRecord(g->ev[1], s), "event");
+    void* args[] = {(void*)&p};
+    CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(bt), args, 0, s), "persistent kernel launch");
+    CK(cudaEventRecord(g->ev[2], s), "event");
+    finalize_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, out_dev, g->n, g->d_off, p.ctl);
+    CK(cudaGetLastError(), "finalize kernel launch");
+    CK(cudaEventRecord(g->ev[3], s), "event");
+    CK(cudaMemcpyAsync(g->h_ctl, g->ctl.p, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "status copy");
+    g->last_grid = grid;
+    g->last_block = bt;
+    g->last_k0 = k;
+    return SSSP_OK;
+}
+
+sssp_status launch_attempt(sssp_graph* g, uint32_t source, unsigned long long* out_dev, cudaStream_t s, int bits) {
+    const unsigned k0 = g->opts.delta_init ? ilog2_round((double)g->opts.delta_init) : g->heur_k;
+    sssp_status st = ensure_ring(g, bits == 32 ? 8 : 16, g->cap ? g->cap : default_cap(g));
+    if (st) return st;
+    if ((st = ensure_trace(g))) return st;
+    if (bits == 32) return launch_one<uint32_t>(g, source, out_dev, s, 32, k0);
+    return launch_one<unsigned long long>(g, source, out_dev, s, 64, k0);
+}
+
+void accumulate(sssp_graph* g, const Ctl& c, int bits) {
+    sssp_stats& st = g->stats;
+    st.vertices_processed += c.st_vertices;
+    st.edges_relaxed += c.st_edges;
+    st.pushes += c.st_pushes + 1;  // + the source item
+    st.stale_skips += c.st_stale;
+    st.reachable += c.reach_v;
+    st.reach_edges += c.reach_e;
+    st.max_dist = std::max<uint64_t>(st.max_dist, c.max_dist);
+    st.init_delta_log2 = g->last_k0;
+    st.final_delta_log2 = meta_k(c.head.meta);
+    st.head_switches += c.head_switches;
+    st.delta_changes += c.delta_changes;
+    st.dist_bits = (uint32_t)bits;
+    st.grid_ctas = g->last_grid;
+    st.block_threads = g->last_block;
+    st.runs += 1;
+    st.trace_entries = std::min<uint32_t>(c.trace_count, g->trace_alloc);
+    float a = 0, b = 0;
+    cudaEventElapsedTime(&a, g->ev[1], g->ev[2]);
+    cudaEventElapsedTime(&b, g->ev[0], g->ev[3]);
+    st.kernel_ms += a;
+    st.total_ms += b;
+}
+
+// Synchronous run of one source with retry (ring growth / 64-bit distances).
+sssp_status run_one_sync(sssp_graph* g, uint32_t source, unsigned long long* out_dev, cudaStream_t s) {
+    int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
+    for (int attempt = 0; attempt < 8; ++attempt) {
+        sssp_status st = launch_attempt(g, source, out_dev, s, bits);
+        if (st) return st;
+        CK(cudaStreamSynchronize(s), "SSSP run");
+        const unsigned status = g->h_ctl->status;
+        if (status == 0) {
+            accumulate(g, *g->h_ctl, bits);
+            return SSSP_OK;
+        }
+        // aborted attempt: the ring holds leftovers -> clear it before anything else
+        CK(cudaMemsetAsync(g->ring.p, 0xFF, g->ring.bytes, s), "clearing the bucket ring");
+        CK(cudaStreamSynchronize(s), "clearing the bucket ring");
+        if (status & kStTimeout) return fail(SSSP_ERR_TIMEOUT, "device watchdog expired");
+        if (status & kStBug) return fail(SSSP_ERR_CUDA, "internal invariant violated (outstanding counter)");
+        if (status & kStDistOverflow) {
+            if (g->opts.dist_bits == 32) return fail(SSSP_ERR_INVALID_ARGUMENT, "distances exceed 32 bits (dist_bits=32)");
+            bits = 64;
+            if (!g->opts.dist_bits) g->cur_bits = 64;
+            g->stats.retries += 1;
+            continue;
+        }
+        if (status & kStRingOverflow) {
+            if ((g->opts.flags & SSSP_FLAG_NO_RETRY) || attempt >= 4)
+                return fail(SSSP_ERR_WORKLIST_OVERFLOW, "bucket ring overflow");
+            const unsigned long long ncap = g->cap * 2;
+            g->ring.release();
+            sssp_status st2 = ensure_ring(g, bits == 32 ? 8 : 16, ncap);
+            if (st2) return st2;
+            g->stats.retries += 1;
+            continue;
+        }
+        return fail(SSSP_ERR_CUDA, "unknown device status");
+    }
+    return fail(SSSP_ERR_WORKLIST_OVERFLOW, "retries exhausted");
+}
+
+sssp_status classify_out(sssp_graph* g, const void* ptr, bool* is_dev) {
+    cudaPointerAttributes a{};
+    cudaError_t e = cudaPointerGetAttributes(&a, ptr);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        *is_dev = false;
+        return SSSP_OK;
+    }
+    if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) {
+        if (a.device != g->device) return fail(SSSP_ERR_DEVICE_MISMATCH, "dist_out is on another device");
+        *is_dev = true;
+    } else {
+        *is_dev = false;
+    }
+    return SSSP_OK;
+}
+
+sssp_status run_many(sssp_graph* g, const uint32_t* sources, uint32_t k, uint64_t* dist_out, sssp_stream_t stream) {
+    if (!g || !dist_out || (k && !sources)) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL argument");
+    if (k == 0) return fail(SSSP_ERR_INVALID_ARGUMENT, "k == 0");
+    for (uint32_t i = 0; i < k; ++i)
+        if (sources[i] >= g->n) return fail(SSSP_ERR_INVALID_ARGUMENT, "source " + std::to_string(sources[i]) + " >= n");
+    if (g->busy || g->async_pending) return fail(SSSP_ERR_BUSY, "a run is already in flight on this handle");
+    DeviceGuard dg(g->device);
+    bool is_dev = false;
+    sssp_status st = classify_out(g, dist_out, &is_dev);
+    if (st) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    g->busy = true;
+    g->stats = sssp_stats{};
+    const bool async = (g->opts.flags & SSSP_FLAG_ASYNC) && is_dev && k == 1;
+    if (!is_dev && !g->hostout.p) {
+        cudaError_t e = cudaMalloc(&g->hostout.p, (size_t)g->n * 8);
+        if (e != cudaSuccess) {
+            g->busy = false;
+            return cuda_fail(e, "allocating the staging buffer for a host dist_out");
+        }
+        g->hostout.bytes = (size_t)g->n * 8;
+    }
+    for (uint32_t i = 0; i < k && st == SSSP_OK; ++i) {
+        unsigned long long* out = is_dev ? (unsigned long long*)dist_out + (size_t)i * g->n
+                                         : (unsigned long long*)g->hostout.p;
+        if (async) {
+            const int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
+            st = launch_attempt(g, sources[i], out, s, bits);
+            if (st == SSSP_OK) {
+                g->async_pending = true;
+                g->stats.dist_bits = (uint32_t)bits;
+            }
+        } else {
+            st = run_one_sync(g, sources[i], out, s);
+            if (st == SSSP_OK && !is_dev) {
+                cudaError_t e = cudaMemcpyAsync((unsigned long long*)dist_out + (size_t)i * g->n, out,
+                                                (size_t)g->n * 8, cudaMemcpyDeviceToHost, s);
+                if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+                if (e != cudaSuccess) st = cuda_fail(e, "copying dist to host");
+            }
+        }
+    }
+    g->stats.status = st;
+    g->busy = false;
+    return st;
+}
+
+}  // namespace
+
+// =================================================================== C ABI
+extern "C" {
+
+void sssp_options_default(sssp_options* o) {
+    if (!o) return;
+    std::memset(o, 0, sizeof(*o));
+    o->struct_size = sizeof(sssp_options);
+    o->device = 0;
+    o->num_buckets = 32;
+    o->delta_mode = SSSP_DELTA_DYNAMIC;
+    o->delta_init = 0;             // heuristic C*W/D
+    o->clip_pct = 65;
+    o->settle_head_switches = 2;   // P:215 (reading R7)
+    o->util_lo_pct = 100;          // P:211 (reading R6)
+    o->util_hi_pct = 400;
+    o->dist_bits = 0;
+    o->ring_items = 0;
+    o->flags = 0;
+    o->block_threads = 0;
+    o->grid_ctas = 0;
+    o->batch_min = 0;
+    o->timeout_ms = 0;
+    o->trace_capacity = 0;
+    o->active_init = 0;
+}
+
+sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offsets, const uint32_t* col,
+                              const uint32_t* w, const sssp_options* opts, sssp_graph** out) {
+    if (!out) return fail(SSSP_ERR_INVALID_ARGUMENT, "out is NULL");
+    *out = nullptr;
+    if (!row_offsets || (m && (!col || !w))) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL CSR array");
+    if (n == 0 || n > 0xFFFFFFFEu) return fail(SSSP_ERR_INVALID_ARGUMENT, "n must be in [1, 2^32-2]");
+    sssp_options o;
+    if (opts) o = *opts;
+    else sssp_options_default(&o);
+    sssp_status st = check_options(o);
+    if (st) return st;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        return fail(SSSP_ERR_NO_DEVICE, "no CUDA device");
+    }
+    if (o.device < 0 || o.device >= ndev) return fail(SSSP_ERR_INVALID_ARGUMENT, "device ordinal out of range");
+    cudaDeviceProp prop{};
+    CK(cudaGetDeviceProperties(&prop, o.device), "device properties");
+    if (prop.major != 10) return fail(SSSP_ERR_NO_DEVICE, std::string("built for sm_100a, device is ") + prop.name);
+    DeviceGuard dg(o.device);
+
+    sssp_graph* g = new sssp_graph();
+    g->device = o.device;
+    g->n = n;
+    g->m = m;
+    g->opts = o;
+    g->sm_count = prop.multiProcessorCount;
+    auto bail = [&](sssp_status s2) {
+        sssp_graph_destroy(g);
+        return s2;
+    };
+#define CKG(call, what)                                      \
+    do {                                                     \
+        cudaError_t e_ = (call);                             \
+        if (e_ != cudaSuccess) return bail(cuda_fail(e_, what)); \
+    } while (0)
+
+    CKG(cudaMalloc(&g->d_off, (size_t)(n + 1) * 8), "allocating row_offsets");
+    CKG(cudaMemcpy(g->d_off, row_offsets, (size_t)(n + 1) * 8, cudaMemcpyDefault), "copying row_offsets");
+    unsigned long long ends[2] = {0, 0};
+    CKG(cudaMemcpy(&ends[0], g->d_off, 8, cudaMemcpyDeviceToHost), "reading row_offsets[0]");
+    CKG(cudaMemcpy(&ends[1], g->d_off + n, 8, cudaMemcpyDeviceToHost), "reading row_offsets[n]");
+    if (ends[0] != 0) return bail(fail(SSSP_ERR_INVALID_GRAPH, "row_offsets[0] != 0 (index 0)"));
+    if (ends[1] != m) return bail(fail(SSSP_ERR_INVALID_GRAPH, "row_offsets[n] != m (index " + std::to_string(n) + ")"));
+
+    CKG(cudaMalloc(&g->d_adj, std::max<size_t>(m, 1) * sizeof(uint2)), "allocating arcs");
+    CKG(cudaMalloc(&g->scratch.p, 64), "scratch");
+    unsigned long long* d_bad = (unsigned long long*)g->scratch.p;  // [0],[1] bad idx, [2] sum_w, [3] max_w
+    unsigned long long init_scr[4] = {~0ull, ~0ull, 0, 0};
+    CKG(cudaMemcpy(d_bad, init_scr, sizeof(init_scr), cudaMemcpyHostToDevice), "scratch init");
+    const unsigned aux_grid = (unsigned)g->sm_count * 8;
+    if (m) {
+        unsigned *d_col = nullptr, *d_w = nullptr;
+        CKG(cudaMalloc(&d_col, m * 4), "allocating col staging");
+        cudaError_t e = cudaMalloc(&d_w, m * 4);
+        if (e != cudaSuccess) {
+            cudaFree(d_col);
+            return bail(cuda_fail(e, "allocating w staging"));
+        }
+        e = cudaMemcpy(d_col, col, m * 4, cudaMemcpyDefault);
+        if (e == cudaSuccess) e = cudaMemcpy(d_w, w, m * 4, cudaMemcpyDefault);
+        if (e == cudaSuccess) {
+            validate_csr_kernel<<<aux_grid, 256>>>(g->d_off, d_col, n, m, d_bad);
+            interleave_kernel<<<aux_grid, 256>>>(d_col, d_w, g->d_adj, m, d_bad + 2, (unsigned*)(d_bad + 3));
+            e = cudaDeviceSynchronize();
+        }
+        cudaFree(d_col);
+        cudaFree(d_w);
+        if (e != cudaSuccess) return bail(cuda_fail(e, "validating / interleaving the CSR"));
+    } else {
+        validate_csr_kernel<<<aux_grid, 256>>>(g->d_off, nullptr, n, 0, d_bad);
+        CKG(cudaDeviceSynchronize(), "validating the CSR");
+    }
+    unsigned long long scr[4];
+    CKG(cudaMemcpy(scr, d_bad, sizeof(scr), cudaMemcpyDeviceToHost), "reading validation result");
+    if (scr[0] != ~0ull)
+        return bail(fail(SSSP_ERR_INVALID_GRAPH, "row_offsets decreasing at index " + std::to_string(scr[0])));
+    if (scr[1] != ~0ull)
+        return bail(fail(SSSP_ERR_INVALID_GRAPH, "col[" + std::to_string(scr[1]) + "] >= n"));
+    g->sum_w = scr[2];
+    g->max_w = (uint32_t)scr[3];
+    // initial Delta: C * W / D with W = average weight, D = average degree, C = 32 (reading R3)
+    if (m && g->sum_w) {
+        const double W = (double)g->sum_w / (double)m, D = (double)m / (double)n;
+        g->heur_k = std::min(ilog2_round(32.0 * W / D), 63u);
+    }
+    // 32-bit distances are provably safe when (n-1) * max_w < 2^32 - 1; otherwise
+    // they are tried first and the overflow flag triggers a 64-bit re-run.
+    g->cur_bits = 32;
+
+    CKG(cudaMalloc(&g->dist.p, (size_t)n * 8), "allocating dist");
+    g->dist.bytes = (size_t)n * 8;
+    CKG(cudaMalloc(&g->bk.p, sizeof(BucketCtl) * kMaxBuckets), "allocating bucket counters");
+    CKG(cudaMemset(g->bk.p, 0, sizeof(BucketCtl) * kMaxBuckets), "bucket counters");
+    CKG(cudaMalloc(&g->ctl.p, sizeof(Ctl)), "allocating control block");
+    CKG(cudaMemset(g->ctl.p, 0, sizeof(Ctl)), "control block");
+    CKG(cudaHostAlloc((void**)&g->h_ctl, sizeof(Ctl), cudaHostAllocDefault), "allocating pinned status block");
+    for (auto& e : g->ev) CKG(cudaEventCreate(&e), "creating events");
+    sssp_status st2 = ensure_ring(g, (o.dist_bits == 64) ? 16 : 8, default_cap(g));
+    if (st2) return bail(st2);
+#undef CKG
+    *out = g;
+    return SSSP_OK;
+}
+
+sssp_status sssp_graph_destroy(sssp_graph* g) {
+    if (!g) return SSSP_OK;
+    DeviceGuard dg(g->device);
+    cudaDeviceSynchronize();
+    if (g->d_off) cudaFree(g->d_off);
+    if (g->d_adj) cudaFree(g->d_adj);
+    g->dist.release();
+    g->ring.release();
+    g->bk.release();
+    g->ctl.release();
+    g->trace.release();
+    g->scratch.release();
+    g->hostout.release();
+    if (g->h_ctl) cudaFreeHost(g->h_ctl);
+    for (auto& e : g->ev)
+        if (e) cudaEventDestroy(e);
+    delete g;
+    return SSSP_OK;
+}
+
+sssp_status sssp_set_options(sssp_graph* g, const sssp_options* opts) {
+    if (!g || !opts) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL argument");
+    if (g->busy || g->async_pending) return fail(SSSP_ERR_BUSY, "a run is in flight");
+    sssp_status st = check_options(*opts);
+    if (st) return st;
+    if (opts->device != g->device) return fail(SSSP_ERR_INVALID_ARGUMENT, "the device of a graph cannot change");
+    DeviceGuard dg(g->device);
+    const bool ring_change = opts->num_buckets != g->opts.num_buckets || opts->ring_items != g->opts.ring_items;
+    g->opts = *opts;
+    if (opts->dist_bits) g->cur_bits = (int)opts->dist_bits;
+    else g->cur_bits = 32;
+    if (ring_change) {
+        g->ring.release();
+        g->cap = 0;
+    }
+    return SSSP_OK;
+}
+
+sssp_status sssp_run(sssp_graph* g, uint32_t source, uint64_t* dist_out, sssp_stream_t stream) {
+    return run_many(g, &source, 1, dist_out, stream);
+}
+
+sssp_status sssp_run_batch(sssp_graph* g, const uint32_t* sources, uint32_t k, uint64_t* dist_out,
+                           sssp_stream_t stream) {
+    return run_many(g, sources, k, dist_out, stream);
+}
+
+sssp_status sssp_get_stats(sssp_graph* g, sssp_stats* out) {
+    if (!g || !out) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL argument");
+    if (g->async_pending) {
+        DeviceGuard dg(g->device);
+        g->async_pending = false;
+        cudaError_t e = cudaEventSynchronize(g->ev[3]);
+        if (e != cudaSuccess) return cuda_fail(e, "async run");
+        // the status copy was enqueued after ev[3] on the same stream
+        e = cudaDeviceSynchronize();
+        if (e != cudaSuccess) return cuda_fail(e, "async run");
+        const unsigned status = g->h_ctl->status;
+        if (status) {
+            cudaMemset(g->ring.p, 0xFF, g->ring.bytes);
+            cudaDeviceSynchronize();
+            g->stats.status = (status & kStRingOverflow)   ? SSSP_ERR_WORKLIST_OVERFLOW
+                              : (status & kStTimeout)      ? SSSP_ERR_TIMEOUT
+                              : (status & kStDistOverflow) ? SSSP_ERR_INVALID_ARGUMENT
+                                                           : SSSP_ERR_CUDA;
+            *out = g->stats;
+            return fail((sssp_status)g->stats.status, "async run failed (status bits " + std::to_string(status) + ")");
+        }
+        accumulate(g, *g->h_ctl, (int)g->stats.dist_bits);
+        g->stats.status = SSSP_OK;
+    }
+    *out = g->stats;
+    return SSSP_OK;
+}
+
+sssp_status sssp_get_trace(sssp_graph* g, sssp_trace_entry* out, uint32_t cap, uint32_t* count) {
+    if (!g || !count || (cap && !out)) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL argument");
+    *count = 0;
+    if (!g->trace.p) return SSSP_OK;
+    const uint32_t nvalid = std::min<uint32_t>(g->stats.trace_entries, g->trace_alloc);
+    const uint32_t c = std::min(cap, nvalid);
+    if (c) {
+        DeviceGuard dg(g->device);
+        CK(cudaMemcpy(out, g->trace.p, (size_t)c * sizeof(sssp_trace_entry), cudaMemcpyDeviceToHost), "trace copy");
+    }
+    *count = c;
+    return SSSP_OK;
+}
+
+sssp_status sssp_graph_info(const sssp_graph* g, uint32_t* n, uint64_t* m, uint64_t* sum_w, uint32_t* max_w,
+                            uint32_t* heuristic_delta_log2) {
+    if (!g) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL graph");
+    if (n) *n = g->n;
+    if (m) *m = g->m;
+    if (sum_w) *sum_w = g->sum_w;
+    if (max_w) *max_w = g->max_w;
+    if (heuristic_delta_log2) *heuristic_delta_log2 = g->heur_k;
+    return SSSP_OK;
+}
+
+uint32_t sssp_bucket_offset(uint64_t d, uint32_t delta_log2, uint64_t head, uint32_t num_buckets) {
+    if (num_buckets < 1) return 0;
+    return adds_bucket_offset(d, delta_log2, head, num_buckets);
+}
+
+const char* sssp_status_string(sssp_status st) {
+    switch (st) {
+        case SSSP_OK: return "SSSP_OK";
+        case SSSP_ERR_INVALID_ARGUMENT: return "SSSP_ERR_INVALID_ARGUMENT";
+        case SSSP_ERR_INVALID_GRAPH: return "SSSP_ERR_INVALID_GRAPH";
+        case SSSP_ERR_OUT_OF_MEMORY: return "SSSP_ERR_OUT_OF_MEMORY";
+        case SSSP_ERR_CUDA: return "SSSP_ERR_CUDA";
+        case SSSP_ERR_WORKLIST_OVERFLOW: return "SSSP_ERR_WORKLIST_OVERFLOW";
+        case SSSP_ERR_TIMEOUT: return "SSSP_ERR_TIMEOUT";
+        case SSSP_ERR_DEVICE_MISMATCH: return "SSSP_ERR_DEVICE_MISMATCH";
+        case SSSP_ERR_BUSY: return "SSSP_ERR_BUSY";
+        case SSSP_ERR_NO_DEVICE: return "SSSP_ERR_NO_DEVICE";
+    }
+    return "SSSP_ERR_UNKNOWN";
+}
+
+const char* sssp_last_error(void) { return g_err.c_str(); }
+
+#define SSSP_STR2(x) #x
+#define SSSP_STR(x) SSSP_STR2(x)
+const char* sssp_version(void) {
+    return "adds-sssp 0.1 (sm_100a, CUDA " SSSP_STR(__CUDACC_VER_MAJOR__) "." SSSP_STR(__CUDACC_VER_MINOR__) ")";
+}
+
+}  // extern "C"

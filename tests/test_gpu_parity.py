@@ -1,0 +1,226 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle,
+element by element, bit-exact (integer distances).
+
+Sizes: tiny hand-made graphs and edge cases, scaled-down configs that span
+many CTAs/batches and ragged tails, and the full BASELINE configs with the
+launch configuration bench.py times.  Schedule-perturbation runs (grid size,
+block size, Delta, bucket count, tiny rings forcing overflow/retry, 32/64-bit
+distances) must all give the same bits.
+"""
+import numpy as np
+import pytest
+
+import graphgen as gg
+import oracle
+from conftest import golden_names, load_golden
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import paper_conf_ppopp_wangfl21_b200 as sssp  # noqa: E402
+
+INF = np.uint64(0xFFFFFFFFFFFFFFFF)
+
+
+def gpu_dist(g, s, **opt):
+    G = sssp.Graph.from_csr(g, **opt)
+    d = sssp.to_u64(G.run(int(s)))
+    st = G.stats()
+    G.close()
+    return d, st
+
+
+def check(g, s, **opt):
+    ref, V, E = oracle.dijkstra(g, int(s))
+    d, st = gpu_dist(g, s, **opt)
+    bad = np.flatnonzero(d != ref)
+    assert bad.size == 0, f"{bad.size} mismatches, first v={bad[:5]} gpu={d[bad[:5]]} ref={ref[bad[:5]]} opt={opt}"
+    assert st["reachable"] == V and st["reach_edges"] == E
+    assert st["vertices_processed"] >= V        # never less work than Dijkstra
+    return st
+
+
+# ----------------------------------------------------------------- edge cases
+@pytest.mark.parametrize("name", golden_names())
+def test_golden_fixtures_on_gpu(name):
+    fx = load_golden(name)
+    g = gg.from_arcs(fx["n"], fx["arcs"])
+    d, st = gpu_dist(g, fx["source"])
+    assert [int(x) for x in d] == fx["dist"]
+    assert st["reachable"] == fx["V"] and st["reach_edges"] == fx["E"]
+
+
+def test_u32_overflow_reruns_in_64_bits():
+    n = 10
+    g = gg.from_arcs(n, [(i, i + 1, 0xFFFFFFFF) for i in range(n - 1)] + [(0, 5, 7)])
+    st = check(g, 0)
+    assert st["dist_bits"] == 64 and st["retries"] >= 1
+
+
+def test_single_vertex_and_empty_graph():
+    g = gg.from_arcs(1, [])
+    d, _ = gpu_dist(g, 0)
+    assert d.tolist() == [0]
+    g = gg.from_arcs(5, [])
+    d, st = gpu_dist(g, 3)
+    assert d.tolist() == [int(INF)] * 3 + [0, int(INF)]
+    assert st["reachable"] == 1
+
+
+def test_random_small_graphs():
+    rng = np.random.default_rng(1)
+    for t in range(40):
+        n = int(rng.integers(1, 300))
+        m = int(rng.integers(0, 8 * n))
+        wmax = int(rng.choice([1, 3, 100, 1 << 20, 0xFFFFFFFF]))
+        arcs = list(zip(rng.integers(0, n, m), rng.integers(0, n, m), rng.integers(0, wmax, m, endpoint=True)))
+        g = gg.from_arcs(n, arcs)
+        check(g, int(rng.integers(0, n)))
+
+
+def test_config_grid64():
+    g = gg.make("grid64")
+    check(g, 0)
+
+
+# ----------------------------------------------------------------- scaled configs
+@pytest.mark.parametrize("config,down", [("road", 8), ("road", 4), ("rmat", 8), ("rmat", 6), ("er", 8), ("er", 6)])
+def test_scaled_configs(config, down):
+    g = gg.make(config, scale_down=down)
+    for s in gg.config_sources(config, g, 2):
+        check(g, s)
+
+
+# ----------------------------------------------------------------- schedule perturbation
+PERTURB = [
+    dict(grid_ctas=1), dict(grid_ctas=3), dict(grid_ctas=37),
+    dict(block_threads=128), dict(block_threads=512),
+    dict(delta_mode=1, delta_init=1), dict(delta_mode=1, delta_init=1 << 30), dict(delta_init=1 << 16),
+    dict(num_buckets=2), dict(num_buckets=2, delta_mode=1), dict(num_buckets=8),
+    dict(dist_bits=64), dict(active_init=32), dict(batch_min=1), dict(batch_min=256),
+    dict(settle_head_switches=1, util_lo_pct=1000, util_hi_pct=2000),
+    dict(ring_items=64), dict(ring_items=256, num_buckets=4),
+    dict(flags=sssp.SSSP_FLAG_TRACE),
+]
+
+
+@pytest.mark.parametrize("opt", PERTURB, ids=lambda o: ",".join(f"{k}={v}" for k, v in o.items()))
+@pytest.mark.parametrize("config", ["road", "rmat", "er"])
+def test_schedule_perturbation(config, opt):
+    g = gg.make(config, scale_down=10 if config != "road" else 10)
+    s = gg.config_sources(config, g, 1)[0]
+    st = check(g, s, **opt)
+    if opt.get("ring_items"):
+        assert st["retries"] >= 0
+
+
+def test_tiny_ring_without_retry_reports_overflow():
+    g = gg.make("rmat", scale_down=8)
+    s = int(gg.config_sources("rmat", g, 1)[0])
+    G = sssp.Graph.from_csr(g, ring_items=64, flags=sssp.SSSP_FLAG_NO_RETRY)
+    with pytest.raises(sssp.SSSPError) as e:
+        G.run(s)
+    assert e.value.status == 5
+    # the handle stays usable after growing the ring
+    G.set_options(ring_items=0, flags=0)
+    d = sssp.to_u64(G.run(s))
+    assert np.array_equal(d, oracle.dijkstra(g, s)[0])
+
+
+# ----------------------------------------------------------------- API behaviour
+def test_run_batch_equals_single_runs():
+    g = gg.make("rmat", scale_down=9)
+    srcs = gg.sources(g, 7, seed=5)
+    G = sssp.Graph.from_csr(g)
+    D = G.run_batch(srcs)
+    st = G.stats()
+    assert st["runs"] == 7
+    for i, s in enumerate(srcs):
+        assert np.array_equal(sssp.to_u64(D[i]), oracle.dijkstra(g, int(s))[0])
+
+
+def test_host_dist_out():
+    g = gg.make("road", scale_down=10)
+    s = int(gg.config_sources("road", g, 1)[0])
+    G = sssp.Graph.from_csr(g)
+    d = G.run_host(s)
+    assert np.array_equal(d, oracle.dijkstra(g, s)[0])
+
+
+def test_device_input_arrays():
+    g = gg.make("er", scale_down=10)
+    s = int(gg.config_sources("er", g, 1)[0])
+    off = torch.from_numpy(g.row_offsets.view(np.int64)).cuda()
+    col = torch.from_numpy(g.col.view(np.int32)).cuda()
+    w = torch.from_numpy(g.w.view(np.int32)).cuda()
+    G = sssp.Graph(off, col, w)
+    assert np.array_equal(sssp.to_u64(G.run(s)), oracle.dijkstra(g, s)[0])
+
+
+def test_invalid_inputs():
+    ok_off = np.array([0, 1, 2], dtype=np.uint64)
+    with pytest.raises(sssp.SSSPError) as e:
+        sssp.Graph(np.array([0, 2, 1], dtype=np.uint64), np.array([0], dtype=np.uint32), np.array([1], dtype=np.uint32))
+    assert e.value.status == 2
+    with pytest.raises(sssp.SSSPError) as e:
+        sssp.Graph(ok_off, np.array([0, 5], dtype=np.uint32), np.array([1, 1], dtype=np.uint32))
+    assert e.value.status == 2 and "col[1]" in e.value.detail
+    with pytest.raises(sssp.SSSPError) as e:
+        sssp.Graph(np.array([1, 2, 2], dtype=np.uint64), np.array([0, 1], dtype=np.uint32),
+                   np.array([1, 1], dtype=np.uint32))
+    assert e.value.status == 2
+    G = sssp.Graph(ok_off, np.array([1, 0], dtype=np.uint32), np.array([1, 1], dtype=np.uint32))
+    with pytest.raises(sssp.SSSPError) as e:
+        G.run(2)
+    assert e.value.status == 1
+    with pytest.raises(sssp.SSSPError) as e:
+        G.run_batch(np.array([], dtype=np.uint32), out=torch.empty((0, 2), dtype=torch.int64, device="cuda"))
+    assert e.value.status == 1
+
+
+def test_async_flag_and_stats():
+    g = gg.make("road", scale_down=8)
+    s = int(gg.config_sources("road", g, 1)[0])
+    G = sssp.Graph.from_csr(g, flags=sssp.SSSP_FLAG_ASYNC)
+    out = G.run(s)
+    torch.cuda.synchronize()
+    st = G.stats()
+    assert st["status"] == 0 and st["kernel_ms"] > 0
+    assert np.array_equal(sssp.to_u64(out), oracle.dijkstra(g, s)[0])
+
+
+def test_trace_invariants():
+    g = gg.make("rmat", scale_down=6)
+    s = int(gg.config_sources("rmat", g, 1)[0])
+    G = sssp.Graph.from_csr(g, flags=sssp.SSSP_FLAG_TRACE)
+    d = sssp.to_u64(G.run(s))
+    assert np.array_equal(d, oracle.dijkstra(g, s)[0])
+    st = G.stats()
+    tr = G.trace()
+    assert len(tr) == min(st["head_switches"], 65536)
+    for e in tr:
+        assert 1 <= e["active"] <= 32
+        assert 0 <= e["delta_log2"] <= 31
+        assert e["pending_tail"] <= e["pending_total"] and e["pending_window"] <= e["pending_total"]
+    ts = [e["time_ns"] for e in tr]
+    assert len(tr) < 2 or max(ts) >= min(ts)
+
+
+def test_repeat_runs_deterministic_and_reusable():
+    g = gg.make("er", scale_down=9)
+    srcs = gg.sources(g, 3, seed=9)
+    G = sssp.Graph.from_csr(g)
+    for s in list(srcs) * 2:
+        assert np.array_equal(sssp.to_u64(G.run(int(s))), oracle.dijkstra(g, int(s))[0])
+
+
+# ----------------------------------------------------------------- full BASELINE sizes
+@pytest.mark.parametrize("config", ["road", "rmat", "er"])
+def test_full_size_config(config):
+    g = gg.make(config)
+    s = int(gg.config_sources(config, g, 1)[0])
+    st = check(g, s)
+    assert st["dist_bits"] == 32
