@@ -163,7 +163,7 @@ sssp_status sssp_set_options(sssp_graph *g, const sssp_options *opts);
  * `source`, UINT64_MAX when unreachable.  Enqueued on `stream`; see
  * "Streams" for the synchronous default and SSSP_FLAG_ASYNC.
  * Errors: INVALID_ARGUMENT (source >= n, NULL dist_out), DEVICE_MISMATCH,
- * BUSY, WORKLIST_OVERFLOW (only with NO_RETRY or after 4 growths), TIMEOUT,
+ * BUSY, WORKLIST_OVERFLOW (only with NO_RETRY or after 20 doublings), TIMEOUT,
  * CUDA. */
 sssp_status sssp_run(sssp_graph *g, uint32_t source, uint64_t *dist_out, sssp_stream_t stream);
 

@@ -264,7 +264,7 @@ void accumulate(sssp_graph* g, const Ctl& c, int bits) {
 // Synchronous run of one source with retry (ring growth / 64-bit distances).
 sssp_status run_one_sync(sssp_graph* g, uint32_t source, unsigned long long* out_dev, cudaStream_t s) {
     int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
-    for (int attempt = 0; attempt < 8; ++attempt) {
+    for (int attempt = 0; attempt < 24; ++attempt) {
         sssp_status st = launch_attempt(g, source, out_dev, s, bits);
         if (st) return st;
         CK(cudaStreamSynchronize(s), "SSSP run");
@@ -286,7 +286,7 @@ sssp_status run_one_sync(sssp_graph* g, uint32_t source, unsigned long long* out
             continue;
         }
         if (status & kStRingOverflow) {
-            if ((g->opts.flags & SSSP_FLAG_NO_RETRY) || attempt >= 4)
+            if ((g->opts.flags & SSSP_FLAG_NO_RETRY) || attempt >= 20)
                 return fail(SSSP_ERR_WORKLIST_OVERFLOW, "bucket ring overflow");
             const unsigned long long ncap = g->cap * 2;
             g->ring.release();
