@@ -68,6 +68,7 @@ typedef enum sssp_status {
 #define SSSP_FLAG_TRACE 0x1u     /* record Delta-controller samples into the trace ring (§5, Figs. 11-15 analog) */
 #define SSSP_FLAG_ASYNC 0x2u     /* do not wait for the run's status block (see Streams above) */
 #define SSSP_FLAG_NO_RETRY 0x4u  /* on worklist overflow return SSSP_ERR_WORKLIST_OVERFLOW instead of growing */
+#define SSSP_FLAG_NO_LOCAL 0x8u  /* publish every child through the ring (ablation of CTA-local continuation) */
 
 /* Delta modes */
 #define SSSP_DELTA_DYNAMIC 0u    /* ADDS: run-time controller */
@@ -95,7 +96,10 @@ typedef struct sssp_options {
     uint32_t timeout_ms;       /* device watchdog (globaltimer); 0 = default 60000 */
     uint32_t trace_capacity;   /* trace ring entries when SSSP_FLAG_TRACE; 0 = 65536 */
     uint32_t active_init;      /* initial number of active (claimable) buckets; 0 = auto (1) */
-    uint32_t reserved[4];
+    uint32_t local_max;        /* head-bucket children a CTA keeps as its own next batch instead of
+                                  publishing them (0 = auto = block_threads; see SSSP_FLAG_NO_LOCAL) */
+    uint32_t max_backoff_ns;   /* idle CTAs back off exponentially up to this (0 = auto = 2048) */
+    uint32_t reserved[2];
 } sssp_options;
 
 typedef struct sssp_stats {

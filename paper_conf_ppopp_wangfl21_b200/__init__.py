@@ -30,6 +30,7 @@ INF = 0xFFFFFFFFFFFFFFFF
 SSSP_FLAG_TRACE = 0x1
 SSSP_FLAG_ASYNC = 0x2
 SSSP_FLAG_NO_RETRY = 0x4
+SSSP_FLAG_NO_LOCAL = 0x8
 SSSP_DELTA_DYNAMIC = 0
 SSSP_DELTA_STATIC = 1
 
@@ -55,7 +56,8 @@ class sssp_options(ctypes.Structure):
         ("util_hi_pct", ctypes.c_uint32), ("dist_bits", ctypes.c_uint32), ("ring_items", ctypes.c_uint64),
         ("flags", ctypes.c_uint32), ("block_threads", ctypes.c_uint32), ("grid_ctas", ctypes.c_uint32),
         ("batch_min", ctypes.c_uint32), ("timeout_ms", ctypes.c_uint32), ("trace_capacity", ctypes.c_uint32),
-        ("active_init", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 4),
+        ("active_init", ctypes.c_uint32), ("local_max", ctypes.c_uint32), ("max_backoff_ns", ctypes.c_uint32),
+        ("reserved", ctypes.c_uint32 * 2),
     ]
 
 

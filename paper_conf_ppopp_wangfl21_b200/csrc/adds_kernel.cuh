@@ -3,31 +3,38 @@
 // One launch runs one single-source SSSP to completion.  Every CTA of the grid
 // is co-resident (cooperative launch) and loops, with no grid-wide barrier:
 //
-//   claim    (§8(a) A4)  warp 0 scans the active
-//            window of the 32-bucket ring (one lane per bucket), picks the
-//            highest-priority bucket with published items and claims a batch
-//            through the bucket's avail gate + claim counter (the decentralised
-//            replacement of the paper's Manager Thread Block, D1).
-//   pop      items are {vertex, distance-at-push}; a slot is empty until its
-//            single 64-bit (or 2x64-bit) store lands, so the item's own store is
-//            its publication (D2; replaces the WCC segments of P:161).
-//            The popper clears the slot behind it.
-//   stale    (A5) an item whose vertex already has a smaller distance is skipped.
+//   claim    (§8(a) A4)  warp 0 reads the status,
+//            the head state and all 32 buckets' avail gates in ONE round trip
+//            (one lane per bucket), picks the highest-priority active bucket
+//            with published items and claims a batch (avail gate, then the
+//            claim counter = read_ptr).  This decentralises the paper's
+//            Manager Thread Block (D1).
+//   pop      items are {vertex, distance-at-push}; a ring slot is empty until
+//            its single 64-bit (2x64-bit) store lands, so the item's own store
+//            is its publication (D2, replaces the WCC segments of
+//            P:161).  The popper clears the slot behind it.
+//   stale    (A5) an item whose vertex already holds a smaller distance is
+//            skipped (checked in parallel with the row-offset loads).
 //   expand   (A5) CTA-cooperative load balancing: exclusive scan of the batch's
-//            degrees, then each thread takes consecutive arcs (coalesced
-//            interleaved {col,w} loads) and finds its owner by binary search.
+//            degrees; each thread takes EPT arcs per round (coalesced 8-byte
+//            {col,w} loads, EPT loads in flight) and finds their owners by
+//            binary search over the scan.
 //   relax    (A6) nd = d + w; a plain L2 load filters, then atomicMin on
 //            dist; the arc improves iff nd < old.
 //   push     (A7) improved vertices go to bucket floor(nd/Delta)
-//            relative to the head, clipped into the tail.  Warp-aggregated
-//            shared-memory staging (ballot + match_any), then one reserve atomic
-//            per (CTA flush, bucket) and coalesced stores into the ring.
-//   complete (A8) done (= CWC) += batch, outstanding -= batch.
+//            relative to the head, clipped into the tail.  Children that land in
+//            the head bucket are kept in shared memory and become this CTA's
+//            next batch (no ring round trip on the dependency chain, DESIGN.md
+//            D3); the rest are staged with warp-aggregated shared-memory
+//            atomics (ballot + match_any), reserved with one atomic per (CTA
+//            flush, bucket) and stored coalesced.
+//   complete (A8) one atomic: done (= CWC) += batch - kept, or
+//            local += kept - batch.
 //   advance  (A8/A9) an idle CTA that sees the head bucket
-//            complete (done == reserve, acquire-ordered) moves the head to the
-//            next non-empty bucket with one 128-bit CAS, running the Delta
-//            controller on the ring's occupancy in the same step.
-//   finish   (A10) outstanding == 0 <=> no item pushed and unfinished.
+//            complete (done == reserve + local, acquire-ordered) moves the head
+//            to the next non-empty bucket with one 128-bit CAS and runs the
+//            Delta controller on the ring occupancy in the same step.
+//   finish   (A10) every bucket complete  <=>  quiescent.
 #pragma once
 #include "bucket_map.h"
 #include "common.cuh"
@@ -57,6 +64,8 @@ struct Params {
     unsigned avg_deg_x16;      // 16 * m / n  ("correlating ... with the average degree")
     unsigned batch_min;
     unsigned share_shift;      // a CTA claims about avail >> share_shift items
+    unsigned local_max;        // head-bucket children a CTA keeps for itself (0 = off)
+    unsigned max_backoff_ns;
     unsigned k_max;
     unsigned long long timeout_ns;
 };
@@ -69,30 +78,34 @@ __device__ __forceinline__ long long warp_sum_s64(long long x) {
     return x;
 }
 
-// --------------------------------------------------------------- head advance
-// Warp-cooperative (lane i <-> ring offset i).  Called by an idle CTA.
+// --------------------------------------------------------------- head advance / termination
+// Warp-cooperative (lane i <-> ring offset i).  Called by an idle CTA's warp 0.
+// Returns true when the whole run is quiescent.
 template <typename DistT>
-__device__ void try_advance(const Params<DistT>& p, const Head hd, const int lane) {
+__device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lane) {
     const unsigned nb = p.nb;
     const unsigned hs = meta_hs(hd.meta), k = meta_k(hd.meta), A = meta_A(hd.meta);
     const unsigned flo = meta_floor(hd.meta), since = meta_since(hd.meta);
     const unsigned slot = (hs + lane) & (nb - 1);
-    long long pend = 0;
+    unsigned long long d = 0, r = 0, l = 0;
+    // every done is read (acquire) before any reserve/local: done(t1) == charged(t2)
+    // with t1 < t2, done <= charged and both monotone  =>  complete at t2
+    if (lane < (int)nb) d = ld_acquire_u64(&p.bk[slot].done.v);
+    __syncwarp();
     if (lane < (int)nb) {
-        // done first (acquire), then reserve: done(t1) == reserve(t2) with t1 < t2
-        // and done <= reserve at all times  =>  the bucket was complete at t2.
-        const unsigned long long d = ld_acquire_u64(&p.bk[slot].done.v);
-        const unsigned long long r = ld_relaxed_u64(&p.bk[slot].reserve.v);
-        pend = (long long)(r - d);
+        r = ld_relaxed_u64(&p.bk[slot].reserve.v);
+        l = ld_relaxed_u64(&p.bk[slot].local.v);
     }
+    const long long pend = (long long)(r + l - d);
+    const long long total = warp_sum_s64(pend);
+    if (total == 0) return true;  // every bucket complete: quiescent
     const long long head_pend = __shfl_sync(FULL, pend, 0);
     const unsigned nz = __ballot_sync(FULL, lane > 0 && lane < (int)nb && pend > 0);
-    if (head_pend != 0 || nz == 0) return;  // head busy, or everything in flight / done
-    const unsigned o = __ffs(nz) - 1;       // first non-empty bucket after the head
-    const long long total = warp_sum_s64(pend);
+    if (head_pend != 0 || nz == 0) return false;  // head busy, or only in-flight work left
+    const unsigned o = __ffs(nz) - 1;              // first non-empty bucket after the head
     const long long tail = __shfl_sync(FULL, pend, nb - 1);
     const long long win = warp_sum_s64((lane >= (int)o && lane < (int)(o + A)) ? pend : 0);
-    if (lane != 0) return;
+    if (lane != 0) return false;
 
     unsigned nk = k, nA = A, nflo = flo, nsince = since + 1;
     bool changed = false;
@@ -143,14 +156,16 @@ __device__ void try_advance(const Params<DistT>& p, const Head hd, const int lan
             }
         }
     }
+    return false;
 }
 
 // --------------------------------------------------------------- kernel
-template <typename DistT, int BT>
+template <typename DistT, int BT, int EPT>
 __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT> p) {
     using IT = ItemT<DistT>;
     using Raw = typename IT::Raw;
-    constexpr int kStage = 2 * BT;  // staged pushes before a forced flush
+    constexpr int kRound = BT * EPT;    // arcs per CTA round
+    constexpr int kStage = 2 * kRound;  // staged pushes before a forced flush
     constexpr int kWarps = BT / 32;
     constexpr unsigned long long kInf = (unsigned long long)DistInf<DistT>::value;
 
@@ -159,112 +174,129 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
     __shared__ unsigned short s_rank[kStage];
     __shared__ unsigned s_cnt[kMaxBuckets];
     __shared__ unsigned long long s_base[kMaxBuckets];
+    __shared__ unsigned s_lv[BT];        // next batch kept locally: vertex
+    __shared__ DistT s_ld[BT];           //                         distance
     __shared__ unsigned long long s_ebeg[BT];
     __shared__ DistT s_d[BT];
     __shared__ unsigned s_scan[BT];
     __shared__ unsigned s_wsum[kWarps];
-    __shared__ unsigned s_total, s_E, s_got, s_slot;
+    __shared__ unsigned s_total, s_E, s_got, s_slot, s_lnext;
     __shared__ int s_cmd;
     __shared__ unsigned long long s_idx;
     __shared__ Head s_head;
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const unsigned nbm = p.nb - 1;
-    unsigned long long c_vert = 0, c_edges = 0, c_push = 0, c_stale = 0;  // thread 0
+    const unsigned local_max = p.local_max < (unsigned)BT ? p.local_max : (unsigned)BT;
+    unsigned long long c_vert = 0, c_edges = 0, c_push = 0, c_stale = 0, c_local = 0;  // thread 0
     unsigned backoff = 0;
+    unsigned have_local = 0;  // uniform: items of the next batch already in s_lv/s_ld
 
     if (tid < (int)kMaxBuckets) s_cnt[tid] = 0;
-    if (tid == 0) s_total = 0;
+    if (tid == 0) {
+        s_total = 0;
+        s_lnext = 0;
+    }
     __syncthreads();
 
     for (;;) {
-        // ------------------------------------------------------------ claim
-        if (warp == 0) {
-            int cmd = CMD_IDLE;
-            unsigned st = 0;
-            if (lane == 0) st = ld_relaxed_u32(&p.ctl->status);
-            st = __shfl_sync(FULL, st, 0);
-            if (st) {
-                cmd = CMD_EXIT;
-            } else {
+        unsigned got, slot;
+        bool from_ring;
+        if (have_local) {
+            got = have_local;
+            slot = s_slot;
+            from_ring = false;
+        } else {
+            // -------------------------------------------------------- claim
+            if (warp == 0) {
+                int cmd = CMD_IDLE;
+                // one round trip: status, head, every bucket's avail gate
+                const unsigned st = ld_relaxed_u32(&p.ctl->status);
                 const Head hd = ld_head(&p.ctl->head);
+                const long long av_abs = lane < (int)p.nb ? (long long)ld_relaxed_u64(&p.bk[lane].avail.v) : 0;
                 const unsigned hs = meta_hs(hd.meta), A = meta_A(hd.meta);
-                const unsigned slot = (hs + lane) & nbm;
-                long long av = 0;
-                if (lane < (int)A) av = (long long)ld_relaxed_u64(&p.bk[slot].avail.v);
-                unsigned mask = __ballot_sync(FULL, av > 0);
-                while (mask) {  // higher-priority buckets first
-                    const int f = __ffs(mask) - 1;
-                    unsigned got = 0;
-                    if (lane == f) {
-                        long long want = av >> p.share_shift;
-                        if (want < (long long)p.batch_min) want = p.batch_min;
-                        if (want > BT) want = BT;
-                        unsigned long long* avp = &p.bk[slot].avail.v;
-                        const long long old = (long long)atomicAdd(avp, (unsigned long long)(-want));
-                        const long long g = old <= 0 ? 0 : (old < want ? old : want);
-                        if (g < want) atomicAdd(avp, (unsigned long long)(want - g));
-                        if (g > 0) {
-                            s_idx = atomicAdd(&p.bk[slot].claim.v, (unsigned long long)g);
-                            s_got = (unsigned)g;
-                            s_slot = slot;
-                            s_head = hd;
+                long long av = __shfl_sync(FULL, av_abs, (hs + lane) & nbm);
+                if (lane >= (int)A) av = 0;
+                if (st) {
+                    cmd = CMD_EXIT;
+                } else {
+                    unsigned mask = __ballot_sync(FULL, av > 0);
+                    while (mask) {  // higher-priority buckets first
+                        const int f = __ffs(mask) - 1;
+                        unsigned g32 = 0;
+                        if (lane == f) {
+                            const unsigned sl = (hs + f) & nbm;
+                            long long want = av >> p.share_shift;
+                            if (want < (long long)p.batch_min) want = p.batch_min;
+                            if (want > BT) want = BT;
+                            unsigned long long* avp = &p.bk[sl].avail.v;
+                            const long long old = (long long)atomicAdd(avp, (unsigned long long)(-want));
+                            const long long g = old <= 0 ? 0 : (old < want ? old : want);
+                            if (g < want) atomicAdd(avp, (unsigned long long)(want - g));
+                            if (g > 0) {
+                                s_idx = atomicAdd(&p.bk[sl].claim.v, (unsigned long long)g);
+                                s_got = (unsigned)g;
+                                s_slot = sl;
+                                s_head = hd;
+                            }
+                            g32 = (unsigned)g;
                         }
-                        got = (unsigned)g;
+                        g32 = __shfl_sync(FULL, g32, f);
+                        if (g32) {
+                            cmd = CMD_WORK;
+                            break;
+                        }
+                        mask &= mask - 1;
                     }
-                    got = __shfl_sync(FULL, got, f);
-                    if (got) {
-                        cmd = CMD_WORK;
-                        break;
-                    }
-                    mask &= mask - 1;
-                }
-                if (cmd != CMD_WORK) {
-                    long long out = 0;
-                    if (lane == 0) out = ld_relaxed_s64(&p.ctl->outstanding);
-                    out = __shfl_sync(FULL, out, 0);
-                    if (out == 0) {
-                        cmd = CMD_EXIT;
-                    } else {
-                        try_advance<DistT>(p, hd, lane);
-                        if (lane == 0) {
+                    if (cmd != CMD_WORK) {
+                        if (try_advance<DistT>(p, hd, lane)) {
+                            cmd = CMD_EXIT;
+                        } else if (lane == 0) {
                             if (globaltimer() - p.ctl->t_start > p.timeout_ns) atomicOr(&p.ctl->status, kStTimeout);
-                            backoff = backoff ? (backoff < 512 ? backoff * 2 : 1024) : 32;
+                            backoff = backoff ? (backoff * 2 < p.max_backoff_ns ? backoff * 2 : p.max_backoff_ns) : 32;
                             __nanosleep(backoff);
                         }
+                    } else if (lane == 0) {
+                        backoff = 0;
                     }
-                } else if (lane == 0) {
-                    backoff = 0;
                 }
+                if (lane == 0) s_cmd = cmd;
             }
-            if (lane == 0) s_cmd = cmd;
+            __syncthreads();
+            const int cmd = s_cmd;
+            if (cmd == CMD_EXIT) break;
+            if (cmd == CMD_IDLE) continue;
+            got = s_got;
+            slot = s_slot;
+            from_ring = true;
         }
-        __syncthreads();
-        const int cmd = s_cmd;
-        if (cmd == CMD_EXIT) break;
-        if (cmd == CMD_IDLE) continue;
 
         // ------------------------------------------------------------ pop + stale check
-        const unsigned got = s_got, slot = s_slot;
         const Head hd = s_head;
         const unsigned hs = meta_hs(hd.meta), k = meta_k(hd.meta);
         unsigned deg = 0;
         bool live = false;
         if (tid < (int)got) {
-            const unsigned long long idx = (s_idx + tid) & (p.cap - 1);
-            char* sp = p.ring + ((size_t)slot * p.cap + idx) * IT::kBytes;
             uint32_t v;
             unsigned long long d;
-            unsigned spins = 0;
-            bool loaded;
-            while (!(loaded = IT::load(sp, v, d))) {  // reserved, store not landed yet
-                if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;  // aborted run
+            bool loaded = true;
+            if (from_ring) {
+                const unsigned long long idx = (s_idx + tid) & (p.cap - 1);
+                char* sp = p.ring + ((size_t)slot * p.cap + idx) * IT::kBytes;
+                unsigned spins = 0;
+                while (!(loaded = IT::load(sp, v, d))) {  // reserved, store not landed yet
+                    if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;  // aborted run
+                }
+                if (loaded) IT::clear(sp);
+            } else {
+                v = s_lv[tid];
+                d = (unsigned long long)s_ld[tid];
             }
             if (loaded) {
-                IT::clear(sp);
+                // the stale check and the row loads are independent: one round trip
                 const unsigned long long cur = (unsigned long long)ld_cg(p.dist + v);
+                const unsigned long long b = p.off[v], e = p.off[v + 1];
                 if (cur >= d) {  // not stale: d is still v's distance ("refined")
-                    const unsigned long long b = p.off[v], e = p.off[v + 1];
                     deg = (unsigned)(e - b);
                     s_ebeg[tid] = b;
                     s_d[tid] = (DistT)d;
@@ -272,6 +304,7 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
                 }
             }
         }
+        if (tid == 0) s_lnext = 0;
         // exclusive scan of degrees over the CTA
         unsigned x = deg;
 #pragma unroll
@@ -303,77 +336,101 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
         }
 
         // ------------------------------------------------------------ expand + relax + push
-        for (unsigned base = 0; base < E; base += BT) {
-            const unsigned e = base + tid;
-            bool push = false;
-            uint32_t pv = 0;
-            unsigned long long pd = 0;
-            if (e < E) {
-                unsigned lo = 0, hi = got - 1;  // owner = largest i with scan[i] <= e
-                while (lo < hi) {
-                    const unsigned mid = (lo + hi + 1) >> 1;
-                    if (s_scan[mid] <= e) lo = mid;
-                    else hi = mid - 1;
+        for (unsigned base = 0; base < E; base += kRound) {
+            unsigned own[EPT];
+            uint2 a[EPT];
+            unsigned long long nd[EPT];
+            bool push[EPT];
+#pragma unroll
+            for (int j = 0; j < EPT; ++j) {
+                const unsigned e = base + j * BT + tid;
+                own[j] = 0;
+                if (e < E) {
+                    unsigned lo = 0, hi = got - 1;  // owner = largest i with scan[i] <= e
+                    while (lo < hi) {
+                        const unsigned mid = (lo + hi + 1) >> 1;
+                        if (s_scan[mid] <= e) lo = mid;
+                        else hi = mid - 1;
+                    }
+                    own[j] = lo;
                 }
-                const uint2 a = __ldg(p.adj + s_ebeg[lo] + (e - s_scan[lo]));
-                const unsigned long long nd = (unsigned long long)s_d[lo] + a.y;
-                if (nd >= kInf) {
-                    atomicOr(&p.ctl->status, kStDistOverflow);  // 32-bit distances insufficient
-                } else {
-                    const DistT cur = ld_cg(p.dist + a.x);
-                    if (nd < (unsigned long long)cur) {
-                        const DistT old = atomicMin(p.dist + a.x, (DistT)nd);
-                        if (nd < (unsigned long long)old) {
-                            push = true;
-                            pv = a.x;
-                            pd = nd;
+            }
+#pragma unroll
+            for (int j = 0; j < EPT; ++j) {  // EPT independent 8-byte arc loads in flight
+                const unsigned e = base + j * BT + tid;
+                a[j] = e < E ? __ldg(p.adj + s_ebeg[own[j]] + (e - s_scan[own[j]])) : make_uint2(0u, 0u);
+            }
+            DistT cur[EPT];
+#pragma unroll
+            for (int j = 0; j < EPT; ++j) {
+                const unsigned e = base + j * BT + tid;
+                nd[j] = (unsigned long long)s_d[own[j]] + a[j].y;
+                cur[j] = (e < E && nd[j] < kInf) ? ld_cg(p.dist + a[j].x) : (DistT)0;
+            }
+#pragma unroll
+            for (int j = 0; j < EPT; ++j) {
+                const unsigned e = base + j * BT + tid;
+                push[j] = false;
+                if (e < E) {
+                    if (nd[j] >= kInf) {
+                        atomicOr(&p.ctl->status, kStDistOverflow);  // 32-bit distances insufficient
+                    } else if (nd[j] < (unsigned long long)cur[j]) {
+                        const DistT old = atomicMin(p.dist + a[j].x, (DistT)nd[j]);
+                        push[j] = nd[j] < (unsigned long long)old;
+                    }
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < EPT; ++j) {
+                const unsigned o = push[j] ? adds_bucket_offset(nd[j], k, hd.h, p.nb) : 0u;
+                // head-bucket children stay in this CTA (warp-aggregated slot grab)
+                bool kept = false;
+                if (local_max) {
+                    const unsigned lm = __ballot_sync(FULL, push[j] && o == 0);
+                    if (lm) {
+                        const int leader = __ffs(lm) - 1;
+                        unsigned pos = 0;
+                        if (lane == leader) pos = atomicAdd(&s_lnext, (unsigned)__popc(lm));
+                        pos = __shfl_sync(FULL, pos, leader) + __popc(lm & lanemask_lt());
+                        if (push[j] && o == 0 && pos < local_max) {
+                            s_lv[pos] = a[j].x;
+                            s_ld[pos] = (DistT)nd[j];
+                            kept = true;
                         }
                     }
                 }
-            }
-            // warp-aggregated staging: one smem atomic per warp for the slot, one
-            // per (warp, bucket) for the rank inside the bucket's run
-            const unsigned act = __ballot_sync(FULL, push);
-            if (push) {
-                const unsigned o = adds_bucket_offset(pd, k, hd.h, p.nb);
-                const int leader = __ffs(act) - 1;
-                unsigned pos = 0;
-                if (lane == leader) pos = atomicAdd(&s_total, (unsigned)__popc(act));
-                pos = __shfl_sync(act, pos, leader) + __popc(act & lanemask_lt());
-                const unsigned peers = __match_any_sync(act, o);
-                const int pl = __ffs(peers) - 1;
-                unsigned r0 = 0;
-                if (lane == pl) r0 = atomicAdd(&s_cnt[o], (unsigned)__popc(peers));
-                r0 = __shfl_sync(peers, r0, pl) + __popc(peers & lanemask_lt());
-                s_items[pos] = IT::make(pv, pd);
-                s_soff[pos] = (unsigned char)o;
-                s_rank[pos] = (unsigned short)r0;
+                const bool pg = push[j] && !kept;
+                const unsigned act = __ballot_sync(FULL, pg);
+                if (pg) {  // warp-aggregated staging for the ring
+                    const int leader = __ffs(act) - 1;
+                    unsigned pos = 0;
+                    if (lane == leader) pos = atomicAdd(&s_total, (unsigned)__popc(act));
+                    pos = __shfl_sync(act, pos, leader) + __popc(act & lanemask_lt());
+                    const unsigned peers = __match_any_sync(act, o);
+                    const int pl = __ffs(peers) - 1;
+                    unsigned r0 = 0;
+                    if (lane == pl) r0 = atomicAdd(&s_cnt[o], (unsigned)__popc(peers));
+                    r0 = __shfl_sync(peers, r0, pl) + __popc(peers & lanemask_lt());
+                    s_items[pos] = IT::make(a[j].x, nd[j]);
+                    s_soff[pos] = (unsigned char)o;
+                    s_rank[pos] = (unsigned short)r0;
+                }
             }
             __syncthreads();
             const unsigned total = s_total;
-            if (total > (unsigned)(kStage - BT) || (base + BT >= E && total > 0)) {
-                // ---------------------------------------------------- flush
-                if (warp == 0) {
-                    if (lane == 0) {
-                        // count children before they become claimable (termination);
-                        // the returned value is consumed, so the add is performed
-                        // before this warp issues the reserves below
-                        const long long before =
-                            (long long)atomicAdd((unsigned long long*)&p.ctl->outstanding, (unsigned long long)total);
-                        if (before <= 0) atomicOr(&p.ctl->status, kStBug);
-                        c_push += total;
-                    }
-                    __syncwarp();
-                    if (lane < (int)p.nb) {
-                        const unsigned c = s_cnt[lane];
-                        if (c) {
-                            const unsigned sl = (hs + lane) & nbm;
-                            const unsigned long long b = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
-                            s_base[lane] = b;
-                            if (b + c > p.cap) {  // lapping: previous occupants must be claimed
-                                const unsigned long long cl = ld_relaxed_u64(&p.bk[sl].claim.v);
-                                if (b + c - p.cap > cl) atomicOr(&p.ctl->status, kStRingOverflow);
-                            }
+            if (total > (unsigned)(kStage - kRound) || (base + kRound >= E && total > 0)) {
+                // ---------------------------------------------------- flush to the ring
+                if (warp == 0 && lane < (int)p.nb) {
+                    const unsigned c = s_cnt[lane];
+                    if (c) {
+                        const unsigned sl = (hs + lane) & nbm;
+                        // returning atomic: the reserve (which also counts the children for
+                        // termination) is performed before this CTA's completion atomic
+                        const unsigned long long b = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
+                        s_base[lane] = b;
+                        if (b + c > p.cap) {  // lapping: previous occupants must be claimed
+                            const unsigned long long cl = ld_relaxed_u64(&p.bk[sl].claim.v);
+                            if (b + c - p.cap > cl) atomicOr(&p.ctl->status, kStRingOverflow);
                         }
                     }
                 }
@@ -403,16 +460,25 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
                         s_cnt[lane] = 0;
                     }
                 }
-                if (tid == 0) s_total = 0;
+                if (tid == 0) {
+                    s_total = 0;
+                    c_push += total;
+                }
                 __syncthreads();
             }
         }
 
         // ------------------------------------------------------------ complete
+        const unsigned kept = s_lnext < local_max ? s_lnext : local_max;
         if (tid == 0) {
-            atomicAdd(&p.bk[slot].done.v, (unsigned long long)got);  // CWC
-            atomicAdd((unsigned long long*)&p.ctl->outstanding, (unsigned long long)(-(long long)got));
+            // one atomic: the kept children inherit the parents' accounting
+            if (got > kept) atomicAdd(&p.bk[slot].done.v, (unsigned long long)(got - kept));
+            else if (kept > got) atomicAdd(&p.bk[slot].local.v, (unsigned long long)(kept - got));
+            c_push += kept;
+            c_local += kept;
         }
+        have_local = kept;
+        if (kept) s_slot = slot;  // (uniform value; every thread writes the same)
         __syncthreads();
     }
 
@@ -421,6 +487,7 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
         atomicAdd(&p.ctl->st_edges, c_edges);
         atomicAdd(&p.ctl->st_pushes, c_push);
         atomicAdd(&p.ctl->st_stale, c_stale);
+        atomicAdd(&p.ctl->st_local, c_local);
     }
 }
 

@@ -54,6 +54,7 @@ __global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned s
             bk[t].avail.v = 0;
             bk[t].claim.v = 0;
             bk[t].done.v = 0;
+            bk[t].local.v = 0;
             if (t == meta_hs(h0.meta)) {  // the source item: bucket 0 = head ("initially ... infinity")
                 IT::store(ring + (size_t)t * cap * IT::kBytes, IT::make(source, 0ull));
                 bk[t].reserve.v = 1;
@@ -62,13 +63,12 @@ __global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned s
         }
         if (t == 0) {
             ctl->head = h0;
-            ctl->outstanding = 1;
             ctl->status = 0;
             ctl->trace_count = 0;
             ctl->head_switches = 0;
             ctl->delta_changes = 0;
             ctl->t_start = globaltimer();
-            ctl->st_vertices = ctl->st_edges = ctl->st_pushes = ctl->st_stale = 0;
+            ctl->st_vertices = ctl->st_edges = ctl->st_pushes = ctl->st_stale = ctl->st_local = 0;
             ctl->reach_v = ctl->reach_e = ctl->max_dist = 0;
         }
     }

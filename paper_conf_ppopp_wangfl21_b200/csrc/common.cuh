@@ -32,7 +32,12 @@ struct BucketCtl {
     Counter avail;    // signed: published and not yet claimed      (claim gate)
     Counter claim;    // items claimed by workers (monotone)        = read_ptr
     Counter done;     // items whose processing completed           = CWC
+    Counter local;    // items kept CTA-local (never stored in the ring) charged to this bucket
 };
+// In flight for bucket b = reserve + local - done.  The bucket is complete when
+// that is 0, and the run is finished when every bucket is complete
+// (exact quiescence, reading R11 of P:182): children are always counted (reserve
+// or local) before their parent's completion is.
 
 // Head state, updated only by 128-bit CAS (one writer per head switch).
 //   h    : absolute number of the head bucket (units of Delta = 2^k)
@@ -64,18 +69,17 @@ struct TraceEntry {  // mirrors sssp_trace_entry
 struct alignas(128) Ctl {
     Head head;
     char pad0_[128 - sizeof(Head)];
-    long long outstanding;  // pushed - completed; 0 <=> quiescent (termination, P:182 reading R11)
-    char pad1_[120];
     unsigned status;
     unsigned trace_count;
     unsigned head_switches;
     unsigned delta_changes;
     unsigned long long t_start;  // %globaltimer at init (watchdog)
     char pad2_[104];
+    unsigned long long st_local;  // items continued CTA-locally
     // statistics (flushed once per CTA at exit, or by finalize)
     unsigned long long st_vertices, st_edges, st_pushes, st_stale;
     unsigned long long reach_v, reach_e, max_dist;
-    unsigned long long pad3_[9];
+    unsigned long long pad3_[8];
 };
 static_assert(sizeof(Ctl) % 128 == 0, "Ctl layout");
 

@@ -118,9 +118,15 @@ sssp_status check_options(const sssp_options& o) {
 }
 
 // ----------------------------------------------------------------- kernel table
+// arcs per thread per round: 4 keeps 4 independent 8-byte loads in flight per
+// thread; halved where the staging buffer would exceed 48 KB of static smem
+template <typename DistT, int BT>
+constexpr int ept() {
+    return (sizeof(DistT) == 8 && BT >= 512) ? 1 : (sizeof(DistT) == 8 || BT >= 512) ? 2 : 4;
+}
 template <typename DistT, int BT>
 void* kfun() {
-    return (void*)adds_persistent_kernel<DistT, BT>;
+    return (void*)adds_persistent_kernel<DistT, BT, ept<DistT, BT>()>;
 }
 void* persistent_fn(int bits, int bt) {
     if (bits == 32) {
@@ -187,6 +193,8 @@ Params<DistT> make_params(sssp_graph* g, unsigned grid, unsigned bt, unsigned k_
     unsigned sh = 0;
     while ((1u << (sh + 1)) <= grid) ++sh;  // floor(log2 grid)
     p.share_shift = sh > 2 ? sh - 2 : 0;
+    p.local_max = (g->opts.flags & SSSP_FLAG_NO_LOCAL) ? 0u : (g->opts.local_max ? g->opts.local_max : bt);
+    p.max_backoff_ns = g->opts.max_backoff_ns ? g->opts.max_backoff_ns : 2048u;
     p.k_max = k_max;
     p.timeout_ns = (unsigned long long)(g->opts.timeout_ms ? g->opts.timeout_ms : 60000u) * 1000000ull;
     return p;
@@ -277,7 +285,7 @@ sssp_status run_one_sync(sssp_graph* g, uint32_t source, unsigned long long* out
         CK(cudaMemsetAsync(g->ring.p, 0xFF, g->ring.bytes, s), "clearing the bucket ring");
         CK(cudaStreamSynchronize(s), "clearing the bucket ring");
         if (status & kStTimeout) return fail(SSSP_ERR_TIMEOUT, "device watchdog expired");
-        if (status & kStBug) return fail(SSSP_ERR_CUDA, "internal invariant violated (outstanding counter)");
+        if (status & kStBug) return fail(SSSP_ERR_CUDA, "internal invariant violated");
         if (status & kStDistOverflow) {
             if (g->opts.dist_bits == 32) return fail(SSSP_ERR_INVALID_ARGUMENT, "distances exceed 32 bits (dist_bits=32)");
             bits = 64;

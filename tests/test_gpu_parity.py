@@ -104,6 +104,7 @@ PERTURB = [
     dict(settle_head_switches=1, util_lo_pct=1000, util_hi_pct=2000),
     dict(ring_items=64), dict(ring_items=256, num_buckets=4),
     dict(flags=sssp.SSSP_FLAG_TRACE),
+    dict(flags=sssp.SSSP_FLAG_NO_LOCAL), dict(local_max=1), dict(local_max=16), dict(max_backoff_ns=64),
 ]
 
 
