@@ -69,6 +69,7 @@ typedef enum sssp_status {
 #define SSSP_FLAG_ASYNC 0x2u     /* do not wait for the run's status block (see Streams above) */
 #define SSSP_FLAG_NO_RETRY 0x4u  /* on worklist overflow return SSSP_ERR_WORKLIST_OVERFLOW instead of growing */
 #define SSSP_FLAG_NO_LOCAL 0x8u  /* publish every child through the ring (ablation of CTA-local continuation) */
+#define SSSP_FLAG_PROFILE 0x10u  /* accumulate per-phase SM-cycle counters (sssp_get_profile) */
 
 /* Delta modes */
 #define SSSP_DELTA_DYNAMIC 0u    /* ADDS: run-time controller */
@@ -187,6 +188,13 @@ sssp_status sssp_get_stats(sssp_graph *g, sssp_stats *out);
 /* Copies up to `cap` trace entries of the last run (SSSP_FLAG_TRACE) into
  * host memory `out`; *count receives the number copied. */
 sssp_status sssp_get_trace(sssp_graph *g, sssp_trace_entry *out, uint32_t cap, uint32_t *count);
+
+/* Per-phase profile of the last run (SSSP_FLAG_PROFILE), summed over CTAs:
+ * out[0..15] = cycles in claim (successful), idle (failed claim + advance +
+ * backoff), pop, scan, rounds (expand/relax/stage), flush, complete, CTA
+ * lifetime; then counts of ring batches, local batches, idle iterations,
+ * flushes, rounds, CTAs; two reserved.  *count receives min(cap, 16). */
+sssp_status sssp_get_profile(sssp_graph *g, uint64_t *out, uint32_t cap, uint32_t *count);
 
 /* Graph facts: n, m, sum of weights, max weight, and the heuristic initial
  * Delta (log2) = round(log2(C * W / D)), C = 32, W = sum_w/m, D = m/n. */

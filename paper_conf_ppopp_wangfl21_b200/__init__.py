@@ -31,6 +31,9 @@ SSSP_FLAG_TRACE = 0x1
 SSSP_FLAG_ASYNC = 0x2
 SSSP_FLAG_NO_RETRY = 0x4
 SSSP_FLAG_NO_LOCAL = 0x8
+SSSP_FLAG_PROFILE = 0x10
+PROFILE_FIELDS = ["cyc_claim", "cyc_idle", "cyc_pop", "cyc_scan", "cyc_rounds", "cyc_flush", "cyc_complete",
+                  "cyc_total", "n_ring_batches", "n_local_batches", "n_idle", "n_flush", "n_rounds", "n_ctas"]
 SSSP_DELTA_DYNAMIC = 0
 SSSP_DELTA_STATIC = 1
 
@@ -93,6 +96,7 @@ SIGNATURES = [
     ("sssp_run_batch", ctypes.c_int, [_P, _P, ctypes.c_uint32, _P, _P]),
     ("sssp_get_stats", ctypes.c_int, [_P, ctypes.POINTER(sssp_stats)]),
     ("sssp_get_trace", ctypes.c_int, [_P, _P, ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint32)]),
+    ("sssp_get_profile", ctypes.c_int, [_P, _P, ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint32)]),
     ("sssp_graph_info", ctypes.c_int, [_P, _P, _P, _P, _P, _P]),
     ("sssp_bucket_offset", ctypes.c_uint32, [ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_uint32]),
     ("sssp_status_string", ctypes.c_char_p, [ctypes.c_int]),
@@ -245,6 +249,12 @@ class Graph:
         cnt = ctypes.c_uint32(0)
         _check(lib().sssp_get_trace(self._h, buf, cap, ctypes.byref(cnt)))
         return [{f: getattr(buf[i], f) for f, _ in sssp_trace_entry._fields_} for i in range(cnt.value)]
+
+    def profile(self) -> dict:
+        buf = (ctypes.c_uint64 * 16)()
+        cnt = ctypes.c_uint32(0)
+        _check(lib().sssp_get_profile(self._h, buf, 16, ctypes.byref(cnt)))
+        return {k: int(buf[i]) for i, k in enumerate(PROFILE_FIELDS)}
 
     def info(self) -> dict:
         n, m, sw, mw, hk = ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_uint32(), ctypes.c_uint32()

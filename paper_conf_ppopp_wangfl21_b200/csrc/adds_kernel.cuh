@@ -66,6 +66,7 @@ struct Params {
     unsigned share_shift;      // a CTA claims about avail >> share_shift items
     unsigned local_max;        // head-bucket children a CTA keeps for itself (0 = off)
     unsigned max_backoff_ns;
+    unsigned prof;             // SSSP_FLAG_PROFILE: accumulate per-phase cycles
     unsigned k_max;
     unsigned long long timeout_ns;
 };
@@ -184,6 +185,7 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
     __shared__ int s_cmd;
     __shared__ unsigned long long s_idx;
     __shared__ Head s_head;
+    __shared__ unsigned long long s_prof[kProfCounters];
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const unsigned nbm = p.nb - 1;
@@ -193,15 +195,20 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
     unsigned have_local = 0;  // uniform: items of the next batch already in s_lv/s_ld
 
     if (tid < (int)kMaxBuckets) s_cnt[tid] = 0;
+    if (tid < (int)kProfCounters) s_prof[tid] = 0;
     if (tid == 0) {
         s_total = 0;
         s_lnext = 0;
     }
+    const bool prof = p.prof != 0 && tid == 0;
+    const long long t_begin = clock64();
+    long long t0 = t_begin, tq = 0;
     __syncthreads();
 
     for (;;) {
         unsigned got, slot;
         bool from_ring;
+        if (prof) t0 = clock64();
         if (have_local) {
             got = have_local;
             slot = s_slot;
@@ -264,6 +271,12 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
             }
             __syncthreads();
             const int cmd = s_cmd;
+            if (prof) {
+                const long long t1 = clock64();
+                s_prof[cmd == CMD_WORK ? PR_CLAIM : PR_IDLE] += t1 - t0;
+                if (cmd == CMD_IDLE) s_prof[PR_N_IDLE] += 1;
+                t0 = t1;
+            }
             if (cmd == CMD_EXIT) break;
             if (cmd == CMD_IDLE) continue;
             got = s_got;
@@ -305,6 +318,12 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
             }
         }
         if (tid == 0) s_lnext = 0;
+        if (prof) {
+            const long long t1 = clock64();
+            s_prof[PR_POP] += t1 - t0;
+            s_prof[from_ring ? PR_N_RING : PR_N_LOCAL] += 1;
+            t0 = t1;
+        }
         // exclusive scan of degrees over the CTA
         unsigned x = deg;
 #pragma unroll
@@ -333,6 +352,12 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
             c_vert += nlive;
             c_stale += got - nlive;
             c_edges += E;
+        }
+        if (prof) {
+            const long long t1 = clock64();
+            s_prof[PR_SCAN] += t1 - t0;
+            t0 = t1;
+            tq = 0;
         }
 
         // ------------------------------------------------------------ expand + relax + push
@@ -418,8 +443,10 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
             }
             __syncthreads();
             const unsigned total = s_total;
+            if (prof) s_prof[PR_N_ROUND] += 1;
             if (total > (unsigned)(kStage - kRound) || (base + kRound >= E && total > 0)) {
                 // ---------------------------------------------------- flush to the ring
+                const long long tf = prof ? clock64() : 0;
                 if (warp == 0 && lane < (int)p.nb) {
                     const unsigned c = s_cnt[lane];
                     if (c) {
@@ -465,7 +492,17 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
                     c_push += total;
                 }
                 __syncthreads();
+                if (prof) {
+                    tq += clock64() - tf;
+                    s_prof[PR_N_FLUSH] += 1;
+                }
             }
+        }
+        if (prof) {
+            const long long t1 = clock64();
+            s_prof[PR_ROUNDS] += t1 - t0 - tq;
+            s_prof[PR_FLUSH] += tq;
+            t0 = t1;
         }
 
         // ------------------------------------------------------------ complete
@@ -480,6 +517,7 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
         have_local = kept;
         if (kept) s_slot = slot;  // (uniform value; every thread writes the same)
         __syncthreads();
+        if (prof) s_prof[PR_COMPLETE] += clock64() - t0;
     }
 
     if (tid == 0) {
@@ -488,6 +526,11 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
         atomicAdd(&p.ctl->st_pushes, c_push);
         atomicAdd(&p.ctl->st_stale, c_stale);
         atomicAdd(&p.ctl->st_local, c_local);
+        if (p.prof) {
+            s_prof[PR_TOTAL] = clock64() - t_begin;
+            s_prof[PR_N_CTAS] = 1;
+            for (int i = 0; i < (int)kProfCounters; ++i) atomicAdd(&p.ctl->prof[i], s_prof[i]);
+        }
     }
 }
 

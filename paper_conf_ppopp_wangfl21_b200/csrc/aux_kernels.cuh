@@ -70,6 +70,7 @@ __global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned s
             ctl->t_start = globaltimer();
             ctl->st_vertices = ctl->st_edges = ctl->st_pushes = ctl->st_stale = ctl->st_local = 0;
             ctl->reach_v = ctl->reach_e = ctl->max_dist = 0;
+            for (int i = 0; i < (int)kProfCounters; ++i) ctl->prof[i] = 0;
         }
     }
 }

@@ -22,6 +22,12 @@ constexpr unsigned kStDistOverflow = 2u;   // 32-bit distance would overflow -> 
 constexpr unsigned kStTimeout = 4u;        // watchdog
 constexpr unsigned kStBug = 8u;            // internal invariant violated
 
+// Phase profile (SSSP_FLAG_PROFILE), summed over CTAs; see sssp_get_profile().
+enum ProfIdx {
+    PR_CLAIM = 0, PR_IDLE, PR_POP, PR_SCAN, PR_ROUNDS, PR_FLUSH, PR_COMPLETE, PR_TOTAL,
+    PR_N_RING, PR_N_LOCAL, PR_N_IDLE, PR_N_FLUSH, PR_N_ROUND, PR_N_CTAS, kProfCounters = 16
+};
+
 struct alignas(128) Counter {
     unsigned long long v;
     unsigned long long pad_[15];
@@ -80,6 +86,7 @@ struct alignas(128) Ctl {
     unsigned long long st_vertices, st_edges, st_pushes, st_stale;
     unsigned long long reach_v, reach_e, max_dist;
     unsigned long long pad3_[8];
+    unsigned long long prof[kProfCounters];  // SSSP_FLAG_PROFILE: per-phase SM cycles / counts (sum over CTAs)
 };
 static_assert(sizeof(Ctl) % 128 == 0, "Ctl layout");
 

@@ -195,6 +195,7 @@ Params<DistT> make_params(sssp_graph* g, unsigned grid, unsigned bt, unsigned k_
     p.share_shift = sh > 2 ? sh - 2 : 0;
     p.local_max = (g->opts.flags & SSSP_FLAG_NO_LOCAL) ? 0u : (g->opts.local_max ? g->opts.local_max : bt);
     p.max_backoff_ns = g->opts.max_backoff_ns ? g->opts.max_backoff_ns : 2048u;
+    p.prof = (g->opts.flags & SSSP_FLAG_PROFILE) ? 1u : 0u;
     p.k_max = k_max;
     p.timeout_ns = (unsigned long long)(g->opts.timeout_ms ? g->opts.timeout_ms : 60000u) * 1000000ull;
     return p;
@@ -591,6 +592,14 @@ sssp_status sssp_get_trace(sssp_graph* g, sssp_trace_entry* out, uint32_t cap, u
         DeviceGuard dg(g->device);
         CK(cudaMemcpy(out, g->trace.p, (size_t)c * sizeof(sssp_trace_entry), cudaMemcpyDeviceToHost), "trace copy");
     }
+    *count = c;
+    return SSSP_OK;
+}
+
+sssp_status sssp_get_profile(sssp_graph* g, uint64_t* out, uint32_t cap, uint32_t* count) {
+    if (!g || !count || (cap && !out)) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL argument");
+    const uint32_t c = std::min<uint32_t>(cap, kProfCounters);
+    for (uint32_t i = 0; i < c; ++i) out[i] = g->h_ctl ? g->h_ctl->prof[i] : 0;
     *count = c;
     return SSSP_OK;
 }

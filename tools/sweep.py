@@ -24,6 +24,7 @@ def main():
     ap.add_argument("--sets", default="[]", help="JSON list of option dicts")
     ap.add_argument("--deltas", default="", help="comma list of log2 Delta for static sweeps")
     ap.add_argument("--extra", default="{}", help="JSON dict merged into every static set")
+    ap.add_argument("--profile", action="store_true", help="add SSSP_FLAG_PROFILE and print phase fractions")
     a = ap.parse_args()
     import torch
     g = gg.make(a.config, scale_down=a.scale_down)
@@ -39,6 +40,8 @@ def main():
         o = sssp.sssp_options_default()
         for kk, v in s.items():
             setattr(o, kk, v)
+        if a.profile:
+            o.flags |= sssp.SSSP_FLAG_PROFILE
         sssp._check(sssp.lib().sssp_set_options(G._h, o))
         G.options = o
         G.run(int(srcs[0]), out=out)  # warm
@@ -50,7 +53,17 @@ def main():
             Eg += st["edges_relaxed"]; Ed += st["reach_edges"]; Vg += st["vertices_processed"]; Vd += st["reachable"]
             dl.append(st["final_delta_log2"])
         ms = statistics.median(ks)
-        print(json.dumps({"config": a.config, "opts": s, "kernel_ms": round(ms, 3),
+        prof = None
+        if a.profile:
+            pr = G.profile()
+            tot = max(1, pr["cyc_total"])
+            prof = {k[4:]: round(v / tot, 3) for k, v in pr.items() if k.startswith("cyc_") and k != "cyc_total"}
+            prof.update({k: v for k, v in pr.items() if k.startswith("n_")})
+            nb = max(1, pr["n_ring_batches"] + pr["n_local_batches"])
+            prof["cyc_per_batch"] = round((pr["cyc_total"] - pr["cyc_idle"]) / nb, 1)
+            prof["rounds_per_batch"] = round(pr["n_rounds"] / nb, 2)
+            prof["items_per_batch"] = round((st["vertices_processed"] + st["stale_skips"]) / nb, 1)
+        print(json.dumps({"prof": prof, "config": a.config, "opts": s, "kernel_ms": round(ms, 3),
                           "gteps": round(Ed / len(srcs) / ms / 1e6, 2), "work_E": round(Eg / Ed, 3),
                           "work_V": round(Vg / Vd, 3), "final_k": dl, "head_switches": st["head_switches"]}),
               flush=True)
