@@ -88,6 +88,14 @@ __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lan
     const unsigned hs = meta_hs(hd.meta), k = meta_k(hd.meta), A = meta_A(hd.meta);
     const unsigned flo = meta_floor(hd.meta), since = meta_since(hd.meta);
     const unsigned slot = (hs + lane) & (nb - 1);
+    // cheap test first: while the head bucket has work in flight there is neither
+    // an advance nor termination to detect (one lane, one round trip)
+    long long hp = 0;
+    if (lane == 0) {
+        const unsigned long long d0 = ld_acquire_u64(&p.bk[hs].done.v);
+        hp = (long long)(ld_relaxed_u64(&p.bk[hs].reserve.v) + ld_relaxed_u64(&p.bk[hs].local.v) - d0);
+    }
+    if (__shfl_sync(FULL, hp, 0) != 0) return false;
     unsigned long long d = 0, r = 0, l = 0;
     // every done is read (acquire) before any reserve/local: done(t1) == charged(t2)
     // with t1 < t2, done <= charged and both monotone  =>  complete at t2
@@ -177,6 +185,8 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
     __shared__ unsigned long long s_base[kMaxBuckets];
     __shared__ unsigned s_lv[BT];        // next batch kept locally: vertex
     __shared__ DistT s_ld[BT];           //                         distance
+    __shared__ unsigned long long s_lbeg[BT];  //                   first arc (prefetched)
+    __shared__ unsigned s_ldeg[BT];      //                         degree (prefetched)
     __shared__ unsigned long long s_ebeg[BT];
     __shared__ DistT s_d[BT];
     __shared__ unsigned s_scan[BT];
@@ -201,6 +211,8 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
         s_lnext = 0;
     }
     const bool prof = p.prof != 0 && tid == 0;
+    const unsigned long long pol_stream = policy_evict_first();  // arcs, row offsets
+    const unsigned long long pol_keep = policy_evict_last();     // dist
     const long long t_begin = clock64();
     long long t0 = t_begin, tq = 0;
     __syncthreads();
@@ -307,8 +319,16 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
             }
             if (loaded) {
                 // the stale check and the row loads are independent: one round trip
-                const unsigned long long cur = (unsigned long long)ld_cg(p.dist + v);
-                const unsigned long long b = p.off[v], e = p.off[v + 1];
+                // (kept children had their row prefetched when they were pushed)
+                const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
+                unsigned long long b, e;
+                if (from_ring) {
+                    b = ld_stream_u64(p.off + v, pol_stream);
+                    e = ld_stream_u64(p.off + v + 1, pol_stream);
+                } else {
+                    b = s_lbeg[tid];
+                    e = b + s_ldeg[tid];
+                }
                 if (cur >= d) {  // not stale: d is still v's distance ("refined")
                     deg = (unsigned)(e - b);
                     s_ebeg[tid] = b;
@@ -383,14 +403,15 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
 #pragma unroll
             for (int j = 0; j < EPT; ++j) {  // EPT independent 8-byte arc loads in flight
                 const unsigned e = base + j * BT + tid;
-                a[j] = e < E ? __ldg(p.adj + s_ebeg[own[j]] + (e - s_scan[own[j]])) : make_uint2(0u, 0u);
+                a[j] = e < E ? ld_stream_u2(p.adj + s_ebeg[own[j]] + (e - s_scan[own[j]]), pol_stream)
+                             : make_uint2(0u, 0u);
             }
             DistT cur[EPT];
 #pragma unroll
             for (int j = 0; j < EPT; ++j) {
                 const unsigned e = base + j * BT + tid;
                 nd[j] = (unsigned long long)s_d[own[j]] + a[j].y;
-                cur[j] = (e < E && nd[j] < kInf) ? ld_cg(p.dist + a[j].x) : (DistT)0;
+                cur[j] = (e < E && nd[j] < kInf) ? ld_keep(p.dist + a[j].x, pol_keep) : (DistT)0;
             }
 #pragma unroll
             for (int j = 0; j < EPT; ++j) {
@@ -400,7 +421,7 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
                     if (nd[j] >= kInf) {
                         atomicOr(&p.ctl->status, kStDistOverflow);  // 32-bit distances insufficient
                     } else if (nd[j] < (unsigned long long)cur[j]) {
-                        const DistT old = atomicMin(p.dist + a[j].x, (DistT)nd[j]);
+                        const DistT old = atomic_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
                         push[j] = nd[j] < (unsigned long long)old;
                     }
                 }
@@ -418,8 +439,14 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
                         if (lane == leader) pos = atomicAdd(&s_lnext, (unsigned)__popc(lm));
                         pos = __shfl_sync(FULL, pos, leader) + __popc(lm & lanemask_lt());
                         if (push[j] && o == 0 && pos < local_max) {
+                            // prefetch the child's row now: its latency overlaps the rest
+                            // of this round instead of the next batch's critical path
+                            const unsigned long long rb = ld_stream_u64(p.off + a[j].x, pol_stream);
+                            const unsigned long long re = ld_stream_u64(p.off + a[j].x + 1, pol_stream);
                             s_lv[pos] = a[j].x;
                             s_ld[pos] = (DistT)nd[j];
+                            s_lbeg[pos] = rb;
+                            s_ldeg[pos] = (unsigned)(re - rb);
                             kept = true;
                         }
                     }

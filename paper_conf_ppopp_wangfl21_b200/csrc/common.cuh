@@ -2,11 +2,12 @@
 //
 // Layout in HBM:
 //   BucketCtl[32]  per ring slot: reserve (P:159 resv_ptr), avail (published -
-//                  claimed gate), claim (P:159 read_ptr), done (P:176 CWC);
+//                  claimed gate), claim (P:159 read_ptr), done (P:176 CWC),
+//                  local (children kept CTA-local);
 //                  every counter on its own 128-B line so the L2 atomic units
 //                  of different counters never serialise on one line.
-//   Ctl            head state (16 B, 128-bit CAS), outstanding-work counter
-//                  (termination), status bits, statistics, trace cursor.
+//   Ctl            head state (16 B, 128-bit CAS), status bits, statistics,
+//                  trace cursor, phase profile.
 //   ring           nb circular arrays of C items each (pre-allocated).
 #pragma once
 #include <cstdint>
@@ -124,6 +125,52 @@ __device__ __forceinline__ void st_relaxed_v2u64(void* p, unsigned long long a, 
 // still a valid upper bound (it only weakens the filter) but L2 is fresher.
 __device__ __forceinline__ unsigned ld_cg(const unsigned* p) { return __ldcg(p); }
 __device__ __forceinline__ unsigned long long ld_cg(const unsigned long long* p) { return __ldcg(p); }
+
+// ---- L2 residency (D5): the arc stream (GBs, read ~once) is marked
+// evict_first so it cannot push the distance array (67/134 MB, gathered and
+// atomically updated at random) out of the 126 MB L2; dist accesses are evict_last.
+__device__ __forceinline__ unsigned long long policy_evict_first() {
+    unsigned long long p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ unsigned long long policy_evict_last() {
+    unsigned long long p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint2 ld_stream_u2(const uint2* a, unsigned long long pol) {
+    uint2 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0, %1}, [%2], %3;"
+                 : "=r"(r.x), "=r"(r.y) : "l"(a), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ unsigned long long ld_stream_u64(const unsigned long long* a, unsigned long long pol) {
+    unsigned long long r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(r) : "l"(a), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ unsigned ld_keep(const unsigned* a, unsigned long long pol) {
+    unsigned r;
+    asm volatile("ld.global.cg.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(a), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ unsigned long long ld_keep(const unsigned long long* a, unsigned long long pol) {
+    unsigned long long r;
+    asm volatile("ld.global.cg.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(r) : "l"(a), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ unsigned atomic_min_keep(unsigned* a, unsigned v, unsigned long long pol) {
+    unsigned r;
+    asm volatile("atom.global.L2::cache_hint.min.u32 %0, [%1], %2, %3;" : "=r"(r) : "l"(a), "r"(v), "l"(pol) : "memory");
+    return r;
+}
+__device__ __forceinline__ unsigned long long atomic_min_keep(unsigned long long* a, unsigned long long v,
+                                                              unsigned long long pol) {
+    unsigned long long r;
+    asm volatile("atom.global.L2::cache_hint.min.u64 %0, [%1], %2, %3;" : "=l"(r) : "l"(a), "l"(v), "l"(pol) : "memory");
+    return r;
+}
 
 __device__ __forceinline__ unsigned long long globaltimer() {
     unsigned long long t;
