@@ -225,3 +225,15 @@ def test_full_size_config(config):
     s = int(gg.config_sources(config, g, 1)[0])
     st = check(g, s)
     assert st["dist_bits"] == 32
+
+
+def test_run_batch_distributed_single_rank():
+    from paper_conf_ppopp_wangfl21_b200.distributed import run_batch_distributed
+    g = gg.make("rmat", scale_down=10)
+    srcs = gg.sources(g, 5, seed=5)
+    G = sssp.Graph.from_csr(g)
+    out = run_batch_distributed(G, srcs, gather=True)
+    full = sssp.to_u64(out["full"])
+    for i, s in enumerate(srcs):
+        assert np.array_equal(full[i], oracle.dijkstra(g, int(s))[0])
+    assert out["stats"]["runs"] == 5
