@@ -70,6 +70,9 @@ typedef enum sssp_status {
 #define SSSP_FLAG_NO_RETRY 0x4u  /* on worklist overflow return SSSP_ERR_WORKLIST_OVERFLOW instead of growing */
 #define SSSP_FLAG_NO_LOCAL 0x8u  /* publish every child through the ring (ablation of CTA-local continuation) */
 #define SSSP_FLAG_PROFILE 0x10u  /* accumulate per-phase SM-cycle counters (sssp_get_profile) */
+#define SSSP_FLAG_NO_L2_PERSIST 0x20u /* do not reserve the L2 persisting set-aside for dist (ablation).
+                                        By default a run raises cudaLimitPersistingL2CacheSize (device-wide)
+                                        up to min(dist bytes, device maximum) */
 
 /* Delta modes */
 #define SSSP_DELTA_DYNAMIC 0u    /* ADDS: run-time controller */
@@ -86,6 +89,11 @@ typedef struct sssp_options {
     uint32_t settle_head_switches; /* K head-bucket switches between Delta changes; default 2 */
     uint32_t util_lo_pct;      /* lower utilisation limit, % of resident threads; default 100 */
     uint32_t util_hi_pct;      /* upper utilisation limit, % of resident threads; default 400 */
+    uint32_t waste_lo_permille;/* Delta may grow only while the recent re-expansion share is below this
+                                  (default 200 = 20%) */
+    uint32_t waste_hi_permille;/* Delta shrinks (not below its clip floor) while the share is above this
+                                  (default 450 = 45%, i.e. ~1.8x Dijkstra's vertex work) */
+    uint32_t period_us;        /* periodic controller step (default 20 us; head switches also step) */
     uint32_t dist_bits;        /* 0 = auto (32-bit internal distances when provably or observably
                                   safe, else 64), 32 or 64 */
     uint64_t ring_items;       /* capacity of each bucket's circular array (items, rounded up to a
@@ -100,7 +108,7 @@ typedef struct sssp_options {
     uint32_t local_max;        /* head-bucket children a CTA keeps as its own next batch instead of
                                   publishing them (0 = auto = block_threads; see SSSP_FLAG_NO_LOCAL) */
     uint32_t max_backoff_ns;   /* idle CTAs back off exponentially up to this (0 = auto = 2048) */
-    uint32_t reserved[2];
+    uint32_t reserved[3];
 } sssp_options;
 
 typedef struct sssp_stats {
@@ -127,15 +135,18 @@ typedef struct sssp_stats {
     uint32_t reserved[3];
 } sssp_stats;
 
-/* One Delta-controller sample (written at each head-bucket switch). */
+/* One Delta-controller sample (written at each head-bucket switch and at each
+ * periodic controller step). */
 typedef struct sssp_trace_entry {
     uint64_t time_ns;        /* %globaltimer */
     uint64_t head;           /* absolute head bucket number */
     uint64_t pending_total;  /* items reserved but not completed, all buckets */
     uint64_t pending_window; /* same, active buckets only */
     uint64_t pending_tail;   /* same, tail (clip) bucket */
-    uint32_t delta_log2;     /* Delta in force after the switch */
-    uint32_t active;         /* active buckets after the switch */
+    uint32_t delta_log2;     /* Delta in force after the step */
+    uint32_t active;         /* active buckets after the step */
+    uint32_t waste_permille; /* re-expansion share of recent expansions (work-waste signal) */
+    uint32_t reason;         /* 1 = head-bucket switch, 2 = periodic controller step */
 } sssp_trace_entry;
 
 /* Opaque handle: owns the device CSR, the workspace (bucket ring, counters,
@@ -193,7 +204,8 @@ sssp_status sssp_get_trace(sssp_graph *g, sssp_trace_entry *out, uint32_t cap, u
  * out[0..15] = cycles in claim (successful), idle (failed claim + advance +
  * backoff), pop, scan, rounds (expand/relax/stage), flush, complete, CTA
  * lifetime; then counts of ring batches, local batches, idle iterations,
- * flushes, rounds, CTAs; two reserved.  *count receives min(cap, 16). */
+ * flushes, rounds, CTAs; then cycles in arc-window setup (owner scan + async
+ * arc prefetch) and the window count.  *count receives min(cap, 16). */
 sssp_status sssp_get_profile(sssp_graph *g, uint64_t *out, uint32_t cap, uint32_t *count);
 
 /* Graph facts: n, m, sum of weights, max weight, and the heuristic initial

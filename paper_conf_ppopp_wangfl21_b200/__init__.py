@@ -32,8 +32,10 @@ SSSP_FLAG_ASYNC = 0x2
 SSSP_FLAG_NO_RETRY = 0x4
 SSSP_FLAG_NO_LOCAL = 0x8
 SSSP_FLAG_PROFILE = 0x10
+SSSP_FLAG_NO_L2_PERSIST = 0x20
 PROFILE_FIELDS = ["cyc_claim", "cyc_idle", "cyc_pop", "cyc_scan", "cyc_rounds", "cyc_flush", "cyc_complete",
-                  "cyc_total", "n_ring_batches", "n_local_batches", "n_idle", "n_flush", "n_rounds", "n_ctas"]
+                  "cyc_total", "n_ring_batches", "n_local_batches", "n_idle", "n_flush", "n_rounds", "n_ctas",
+                  "cyc_window", "n_windows"]
 SSSP_DELTA_DYNAMIC = 0
 SSSP_DELTA_STATIC = 1
 
@@ -56,11 +58,13 @@ class sssp_options(ctypes.Structure):
         ("struct_size", ctypes.c_uint32), ("device", ctypes.c_int32), ("num_buckets", ctypes.c_uint32),
         ("delta_mode", ctypes.c_uint32), ("delta_init", ctypes.c_uint64), ("clip_pct", ctypes.c_uint32),
         ("settle_head_switches", ctypes.c_uint32), ("util_lo_pct", ctypes.c_uint32),
-        ("util_hi_pct", ctypes.c_uint32), ("dist_bits", ctypes.c_uint32), ("ring_items", ctypes.c_uint64),
+        ("util_hi_pct", ctypes.c_uint32), ("waste_lo_permille", ctypes.c_uint32),
+        ("waste_hi_permille", ctypes.c_uint32), ("period_us", ctypes.c_uint32),
+        ("dist_bits", ctypes.c_uint32), ("ring_items", ctypes.c_uint64),
         ("flags", ctypes.c_uint32), ("block_threads", ctypes.c_uint32), ("grid_ctas", ctypes.c_uint32),
         ("batch_min", ctypes.c_uint32), ("timeout_ms", ctypes.c_uint32), ("trace_capacity", ctypes.c_uint32),
         ("active_init", ctypes.c_uint32), ("local_max", ctypes.c_uint32), ("max_backoff_ns", ctypes.c_uint32),
-        ("reserved", ctypes.c_uint32 * 2),
+        ("reserved", ctypes.c_uint32 * 3),
     ]
 
 
@@ -80,7 +84,7 @@ class sssp_trace_entry(ctypes.Structure):
     _fields_ = [
         ("time_ns", ctypes.c_uint64), ("head", ctypes.c_uint64), ("pending_total", ctypes.c_uint64),
         ("pending_window", ctypes.c_uint64), ("pending_tail", ctypes.c_uint64), ("delta_log2", ctypes.c_uint32),
-        ("active", ctypes.c_uint32),
+        ("active", ctypes.c_uint32), ("waste_permille", ctypes.c_uint32), ("reason", ctypes.c_uint32),
     ]
 
 

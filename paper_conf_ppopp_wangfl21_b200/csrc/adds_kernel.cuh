@@ -67,6 +67,10 @@ struct Params {
     unsigned local_max;        // head-bucket children a CTA keeps for itself (0 = off)
     unsigned max_backoff_ns;
     unsigned prof;             // SSSP_FLAG_PROFILE: accumulate per-phase cycles
+    float keep_frac;           // fraction of dist covered by the L2 persisting set-aside
+    unsigned* expanded;        // n-bit bitmap: vertex expanded at least once (controller waste signal)
+    unsigned waste_lo, waste_hi;  // permille
+    unsigned long long period_ns;
     unsigned k_max;
     unsigned long long timeout_ns;
 };
@@ -79,15 +83,120 @@ __device__ __forceinline__ long long warp_sum_s64(long long x) {
     return x;
 }
 
+// --------------------------------------------------------------- Delta controller
+// P:205-217 (§5.5).  Inputs, read warp-cooperatively (lane i <-> ring offset i):
+// pending items per bucket (reserved + kept - done), hence the head, the active
+// window (utilisation = window items x average degree vs resident threads,
+// P:211) and the tail (clip share); plus the recent re-expansion
+// share of expansions (work-waste signal, R6).  Readings:
+//   clip   tail >= clip_pct of all pending        -> Delta x2, floor = Delta
+//   waste  share > waste_hi after settling        -> Delta /2 (not below floor)
+//   grow   window under-utilised AND share < lo   -> Delta x2
+//   A      active buckets follow the same two signals one step at a time
+// Settling: `since` counts controller steps (head switches and periodic
+// steps) since the last Delta change; a change needs since >= settle.
+struct CtlDecision {
+    unsigned k, A, flo, since;
+    bool changed;
+};
+
+template <typename DistT>
+__device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, unsigned flo, unsigned since,
+                              long long total, long long tail, long long win, unsigned waste, bool waste_known) {
+    CtlDecision d{k, A, flo, since + 1, false};
+    if (!p.dynamic) return d;
+    const unsigned long long util = ((unsigned long long)(win > 0 ? win : 0) * p.avg_deg_x16) >> 4;
+    const unsigned long long T = p.resident_threads;
+    const bool low = util * 100ull < (unsigned long long)p.util_lo_pct * T;
+    const bool high = util * 100ull > (unsigned long long)p.util_hi_pct * T;
+    const bool wasteful = waste_known && waste > p.waste_hi;
+    const bool frugal = waste_known && waste < p.waste_lo;
+    if (total >= 64 && tail * 100 >= (long long)p.clip_pct * total && k < p.k_max) {
+        d.k = k + 1;  // clipping: raise Delta and its lower bound
+        d.flo = d.k;
+        d.changed = true;
+    } else if (d.since >= p.settle) {
+        if (wasteful && k > flo) {
+            d.k = k - 1;
+            d.changed = true;
+        } else if (low && frugal && k < p.k_max) {
+            d.k = k + 1;
+            d.changed = true;
+        }
+    }
+    if (d.changed) d.since = 0;
+    if (low && frugal && A < p.nb) d.A = A + 1;
+    else if ((wasteful || high) && A > 1) d.A = A - 1;
+    return d;
+}
+
+// Pending items of the 32 buckets relative to the head (acquire-ordered so that a
+// zero really means complete): every done is read before any reserve/local.
+template <typename DistT>
+__device__ __forceinline__ long long bucket_pending(const Params<DistT>& p, unsigned hs, int lane) {
+    const unsigned slot = (hs + lane) & (p.nb - 1);
+    unsigned long long d = 0, r = 0, l = 0;
+    if (lane < (int)p.nb) d = ld_acquire_u64(&p.bk[slot].done.v);
+    __syncwarp();
+    if (lane < (int)p.nb) {
+        r = ld_relaxed_u64(&p.bk[slot].reserve.v);
+        l = ld_relaxed_u64(&p.bk[slot].local.v);
+    }
+    return (long long)(r + l - d);
+}
+
+template <typename DistT>
+__device__ __forceinline__ unsigned recent_waste(const Params<DistT>& p, bool& known) {
+    const unsigned long long e = ld_relaxed_u64(&p.ctl->g_exp) - ld_relaxed_u64(&p.ctl->exp_mark);
+    const unsigned long long f = ld_relaxed_u64(&p.ctl->g_first) - ld_relaxed_u64(&p.ctl->first_mark);
+    known = e >= 4096;
+    return (known && e > f) ? (unsigned)((e - f) * 1000ull / e) : 0u;
+}
+
+// Commit a controller step by 128-bit CAS; restart the waste window on a change
+// (and every 8 steps so the signal tracks the recent past).
+template <typename DistT>
+__device__ void commit_step(const Params<DistT>& p, const Head hd, const Head nhd, bool kchanged, unsigned since,
+                            long long total, long long win, long long tail, unsigned waste, unsigned reason) {
+    Head seen;
+    if (!cas_head(&p.ctl->head, hd, nhd, seen)) return;
+    if (reason == 1) atomicAdd(&p.ctl->head_switches, 1u);
+    if (kchanged) atomicAdd(&p.ctl->delta_changes, 1u);
+    if (kchanged || (since & 7) == 0) {
+        p.ctl->exp_mark = ld_relaxed_u64(&p.ctl->g_exp);
+        p.ctl->first_mark = ld_relaxed_u64(&p.ctl->g_first);
+    }
+    if (p.trace_cap) {
+        const unsigned t = atomicAdd(&p.ctl->trace_count, 1u);
+        if (t < p.trace_cap) {
+            TraceEntry e;
+            e.time_ns = globaltimer();
+            e.head = nhd.h;
+            e.pending_total = (unsigned long long)total;
+            e.pending_window = (unsigned long long)win;
+            e.pending_tail = (unsigned long long)tail;
+            e.delta_log2 = meta_k(nhd.meta);
+            e.active = meta_A(nhd.meta);
+            e.waste_permille = waste;
+            e.reason = reason;
+            p.trace[t] = e;
+        }
+    }
+}
+
+// Re-express the absolute head bucket number under a new Delta exponent.
+__device__ __forceinline__ unsigned long long rehead(unsigned long long h, unsigned k, unsigned nk) {
+    if (nk > k) return h >> (nk - k);
+    if (nk < k) return h << (k - nk);
+    return h;
+}
+
 // --------------------------------------------------------------- head advance / termination
-// Warp-cooperative (lane i <-> ring offset i).  Called by an idle CTA's warp 0.
-// Returns true when the whole run is quiescent.
+// Called by an idle CTA's warp 0.  Returns true when the whole run is quiescent.
 template <typename DistT>
 __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lane) {
     const unsigned nb = p.nb;
     const unsigned hs = meta_hs(hd.meta), k = meta_k(hd.meta), A = meta_A(hd.meta);
-    const unsigned flo = meta_floor(hd.meta), since = meta_since(hd.meta);
-    const unsigned slot = (hs + lane) & (nb - 1);
     // cheap test first: while the head bucket has work in flight there is neither
     // an advance nor termination to detect (one lane, one round trip)
     long long hp = 0;
@@ -96,18 +205,9 @@ __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lan
         hp = (long long)(ld_relaxed_u64(&p.bk[hs].reserve.v) + ld_relaxed_u64(&p.bk[hs].local.v) - d0);
     }
     if (__shfl_sync(FULL, hp, 0) != 0) return false;
-    unsigned long long d = 0, r = 0, l = 0;
-    // every done is read (acquire) before any reserve/local: done(t1) == charged(t2)
-    // with t1 < t2, done <= charged and both monotone  =>  complete at t2
-    if (lane < (int)nb) d = ld_acquire_u64(&p.bk[slot].done.v);
-    __syncwarp();
-    if (lane < (int)nb) {
-        r = ld_relaxed_u64(&p.bk[slot].reserve.v);
-        l = ld_relaxed_u64(&p.bk[slot].local.v);
-    }
-    const long long pend = (long long)(r + l - d);
+    const long long pend = bucket_pending(p, hs, lane);
     const long long total = warp_sum_s64(pend);
-    if (total == 0) return true;  // every bucket complete: quiescent
+    if (total == 0) return true;  // every bucket complete: quiescent (reading R11)
     const long long head_pend = __shfl_sync(FULL, pend, 0);
     const unsigned nz = __ballot_sync(FULL, lane > 0 && lane < (int)nb && pend > 0);
     if (head_pend != 0 || nz == 0) return false;  // head busy, or only in-flight work left
@@ -115,81 +215,81 @@ __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lan
     const long long tail = __shfl_sync(FULL, pend, nb - 1);
     const long long win = warp_sum_s64((lane >= (int)o && lane < (int)(o + A)) ? pend : 0);
     if (lane != 0) return false;
-
-    unsigned nk = k, nA = A, nflo = flo, nsince = since + 1;
-    bool changed = false;
-    if (p.dynamic) {
-        // utilisation = edge work available in the active window
-        const unsigned long long util = ((unsigned long long)win * p.avg_deg_x16) >> 4;
-        const unsigned long long T = p.resident_threads;
-        const bool low = util * 100ull < (unsigned long long)p.util_lo_pct * T;
-        const bool high = util * 100ull > (unsigned long long)p.util_hi_pct * T;
-        if (total >= 64 && tail * 100 >= (long long)p.clip_pct * total && nk < p.k_max) {
-            nk = k + 1;  // clipping: raise Delta and its lower bound
-            nflo = nk;
-            changed = true;
-        } else if (nsince >= p.settle) {  // settle for K head switches
-            if (low && nk < p.k_max) {
-                nk = k + 1;
-                changed = true;
-            } else if (high && nk > nflo) {
-                nk = k - 1;
-                changed = true;
-            }
-        }
-        if (changed) nsince = 0;
-        // fine-grained knob: number of active buckets
-        if (low && nA < nb) nA = nA + 1;
-        else if (high && nA > 1) nA = nA - 1;
-    }
-    unsigned long long nh = hd.h + o;
-    if (nk > k) nh >>= (nk - k);
-    else if (nk < k) nh <<= (k - nk);
-    const Head nhd{nh, pack_meta((hs + o) & (nb - 1), nk, nA, nflo, nsince > 0xffff ? 0xffff : nsince)};
-    Head seen;
-    if (cas_head(&p.ctl->head, hd, nhd, seen)) {
-        atomicAdd(&p.ctl->head_switches, 1u);
-        if (nk != k) atomicAdd(&p.ctl->delta_changes, 1u);
-        if (p.trace_cap) {
-            const unsigned t = atomicAdd(&p.ctl->trace_count, 1u);
-            if (t < p.trace_cap) {
-                TraceEntry e;
-                e.time_ns = globaltimer();
-                e.head = nh;
-                e.pending_total = (unsigned long long)total;
-                e.pending_window = (unsigned long long)win;
-                e.pending_tail = (unsigned long long)tail;
-                e.delta_log2 = nk;
-                e.active = nA;
-                p.trace[t] = e;
-            }
-        }
-    }
+    bool known;
+    const unsigned waste = recent_waste(p, known);
+    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), total, tail, win, waste, known);
+    const Head nhd{rehead(hd.h + o, k, d.k),
+                   pack_meta((hs + o) & (nb - 1), d.k, d.A, d.flo, d.since > 0xffff ? 0xffff : d.since)};
+    commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 1u);
     return false;
 }
 
+// Periodic controller step ("the MTB periodically gathers run-time
+// information"), run by warp 0 of a CTA that won the period.  The head stays
+// where it is; only its number is re-expressed if Delta changes.
+template <typename DistT>
+__device__ void periodic_step(const Params<DistT>& p, const int lane) {
+    const Head hd = ld_head(&p.ctl->head);
+    const unsigned hs = meta_hs(hd.meta), k = meta_k(hd.meta), A = meta_A(hd.meta);
+    const long long pend = bucket_pending(p, hs, lane);
+    const long long total = warp_sum_s64(pend);
+    const long long tail = __shfl_sync(FULL, pend, p.nb - 1);
+    const long long win = warp_sum_s64(lane < (int)A ? pend : 0);
+    if (lane != 0 || total == 0) return;
+    bool known;
+    const unsigned waste = recent_waste(p, known);
+    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), total, tail, win, waste, known);
+    const Head nhd{rehead(hd.h, k, d.k), pack_meta(hs, d.k, d.A, d.flo, d.since > 0xffff ? 0xffff : d.since)};
+    commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 2u);
+}
+
+// --------------------------------------------------------------- shared memory
+constexpr size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
+
+template <typename DistT, int BT, int EPT, int W>
+struct Smem {
+    using Raw = typename ItemT<DistT>::Raw;
+    static constexpr int kStage = 2 * BT * EPT;  // staged ring pushes before a forced flush
+    static constexpr size_t o_arc = 0;                                        // uint2[W]   arc window
+    static constexpr size_t o_items = o_arc + (size_t)W * 8;                  // Raw[kStage] staged pushes
+    static constexpr size_t o_ebeg = o_items + align16((size_t)kStage * sizeof(Raw));  // u64[BT] row begin
+    static constexpr size_t o_d = o_ebeg + (size_t)BT * 8;                    // DistT[BT]  item distance
+    static constexpr size_t o_ld = o_d + align16((size_t)BT * sizeof(DistT)); // DistT[BT]  kept children
+    static constexpr size_t o_owner = o_ld + align16((size_t)BT * sizeof(DistT));  // u16[W] arc -> item
+    static constexpr size_t o_rank = o_owner + align16((size_t)W * 2);        // u16[kStage]
+    static constexpr size_t o_scan = o_rank + align16((size_t)kStage * 2);    // u32[BT]
+    static constexpr size_t o_lv = o_scan + align16((size_t)BT * 4);          // u32[BT] kept children
+    static constexpr size_t o_soff = o_lv + align16((size_t)BT * 4);          // u8[kStage]
+    static constexpr size_t bytes = o_soff + align16((size_t)kStage);
+};
+
 // --------------------------------------------------------------- kernel
-template <typename DistT, int BT, int EPT>
-__global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT> p) {
+template <typename DistT, int BT, int EPT, int W>
+__global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Params<DistT> p) {
     using IT = ItemT<DistT>;
     using Raw = typename IT::Raw;
-    constexpr int kRound = BT * EPT;    // arcs per CTA round
-    constexpr int kStage = 2 * kRound;  // staged pushes before a forced flush
+    using L = Smem<DistT, BT, EPT, W>;
+    constexpr int kStage = L::kStage;
+    constexpr int kRound = BT * EPT;  // arcs per CTA round
     constexpr int kWarps = BT / 32;
+    constexpr int kPer = W / BT;      // window positions per thread in the owner scan
     constexpr unsigned long long kInf = (unsigned long long)DistInf<DistT>::value;
+    static_assert(W % BT == 0 && kPer >= 1, "window");
 
-    __shared__ Raw s_items[kStage];
-    __shared__ unsigned char s_soff[kStage];
-    __shared__ unsigned short s_rank[kStage];
+    extern __shared__ __align__(16) unsigned char smem[];
+    uint2* s_arc = (uint2*)(smem + L::o_arc);
+    Raw* s_items = (Raw*)(smem + L::o_items);
+    unsigned long long* s_ebeg = (unsigned long long*)(smem + L::o_ebeg);
+    DistT* s_d = (DistT*)(smem + L::o_d);
+    DistT* s_ld = (DistT*)(smem + L::o_ld);
+    unsigned short* s_owner = (unsigned short*)(smem + L::o_owner);
+    unsigned short* s_rank = (unsigned short*)(smem + L::o_rank);
+    unsigned* s_scan = (unsigned*)(smem + L::o_scan);
+    unsigned* s_lv = (unsigned*)(smem + L::o_lv);
+    unsigned char* s_soff = (unsigned char*)(smem + L::o_soff);
+
     __shared__ unsigned s_cnt[kMaxBuckets];
     __shared__ unsigned long long s_base[kMaxBuckets];
-    __shared__ unsigned s_lv[BT];        // next batch kept locally: vertex
-    __shared__ DistT s_ld[BT];           //                         distance
-    __shared__ unsigned long long s_lbeg[BT];  //                   first arc (prefetched)
-    __shared__ unsigned s_ldeg[BT];      //                         degree (prefetched)
-    __shared__ unsigned long long s_ebeg[BT];
-    __shared__ DistT s_d[BT];
-    __shared__ unsigned s_scan[BT];
     __shared__ unsigned s_wsum[kWarps];
     __shared__ unsigned s_total, s_E, s_got, s_slot, s_lnext;
     __shared__ int s_cmd;
@@ -198,6 +298,8 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
     __shared__ unsigned long long s_prof[kProfCounters];
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const unsigned lt_mask = lanemask_lt();
+    const unsigned s_arc_addr = smem_addr(s_arc);
     const unsigned nbm = p.nb - 1;
     const unsigned local_max = p.local_max < (unsigned)BT ? p.local_max : (unsigned)BT;
     unsigned long long c_vert = 0, c_edges = 0, c_push = 0, c_stale = 0, c_local = 0;  // thread 0
@@ -212,9 +314,9 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
     }
     const bool prof = p.prof != 0 && tid == 0;
     const unsigned long long pol_stream = policy_evict_first();  // arcs, row offsets
-    const unsigned long long pol_keep = policy_evict_last();     // dist
+    const unsigned long long pol_keep = policy_evict_last(p.keep_frac);  // dist
     const long long t_begin = clock64();
-    long long t0 = t_begin, tq = 0;
+    long long t0 = t_begin, tq = 0, tw = 0;
     __syncthreads();
 
     for (;;) {
@@ -300,7 +402,7 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
         const Head hd = s_head;
         const unsigned hs = meta_hs(hd.meta), k = meta_k(hd.meta);
         unsigned deg = 0;
-        bool live = false;
+        bool live = false, first = false;
         if (tid < (int)got) {
             uint32_t v;
             unsigned long long d;
@@ -319,21 +421,18 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
             }
             if (loaded) {
                 // the stale check and the row loads are independent: one round trip
-                // (kept children had their row prefetched when they were pushed)
                 const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
-                unsigned long long b, e;
-                if (from_ring) {
-                    b = ld_stream_u64(p.off + v, pol_stream);
-                    e = ld_stream_u64(p.off + v + 1, pol_stream);
-                } else {
-                    b = s_lbeg[tid];
-                    e = b + s_ldeg[tid];
-                }
+                const unsigned long long b = ld_stream_u64(p.off + v, pol_stream);
+                const unsigned long long e = ld_stream_u64(p.off + v + 1, pol_stream);
                 if (cur >= d) {  // not stale: d is still v's distance ("refined")
                     deg = (unsigned)(e - b);
                     s_ebeg[tid] = b;
                     s_d[tid] = (DistT)d;
                     live = true;
+                    if (p.dynamic) {  // work-waste signal: is this v's first expansion?
+                        const unsigned bit = 1u << (v & 31);
+                        first = (atomicOr(p.expanded + (v >> 5), bit) & bit) == 0;
+                    }
                 }
             }
         }
@@ -353,6 +452,7 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
         }
         if (lane == 31) s_wsum[warp] = x;
         const int nlive = __syncthreads_count(live);
+        const int nfirst = p.dynamic ? __syncthreads_count(first) : 0;
         if (warp == 0) {
             const unsigned ws = lane < kWarps ? s_wsum[lane] : 0;
             unsigned inc = ws;
@@ -367,7 +467,6 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
         __syncthreads();
         s_scan[tid] = x - deg + s_wsum[warp];
         const unsigned E = s_E;
-        __syncthreads();
         if (tid == 0) {
             c_vert += nlive;
             c_stale += got - nlive;
@@ -378,161 +477,214 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
             s_prof[PR_SCAN] += t1 - t0;
             t0 = t1;
             tq = 0;
+            tw = 0;
         }
 
-        // ------------------------------------------------------------ expand + relax + push
-        for (unsigned base = 0; base < E; base += kRound) {
-            unsigned own[EPT];
-            uint2 a[EPT];
-            unsigned long long nd[EPT];
-            bool push[EPT];
+        for (unsigned wbase = 0; wbase < E; wbase += W) {
+            const unsigned Ew = (E - wbase) < (unsigned)W ? (E - wbase) : (unsigned)W;
+            const long long tw0 = prof ? clock64() : 0;
+            // ------------------------------------------------ owner of every window position
+            // zero, mark row starts, inclusive prefix-max (rows are in scan order)
+            {
+                unsigned short* ow = s_owner + tid * kPer;
 #pragma unroll
-            for (int j = 0; j < EPT; ++j) {
-                const unsigned e = base + j * BT + tid;
-                own[j] = 0;
-                if (e < E) {
-                    unsigned lo = 0, hi = got - 1;  // owner = largest i with scan[i] <= e
-                    while (lo < hi) {
-                        const unsigned mid = (lo + hi + 1) >> 1;
-                        if (s_scan[mid] <= e) lo = mid;
-                        else hi = mid - 1;
-                    }
-                    own[j] = lo;
-                }
+                for (int i = 0; i < kPer; ++i) ow[i] = 0;
             }
-#pragma unroll
-            for (int j = 0; j < EPT; ++j) {  // EPT independent 8-byte arc loads in flight
-                const unsigned e = base + j * BT + tid;
-                a[j] = e < E ? ld_stream_u2(p.adj + s_ebeg[own[j]] + (e - s_scan[own[j]]), pol_stream)
-                             : make_uint2(0u, 0u);
+            __syncthreads();  // (also publishes s_scan)
+            if (tid < (int)got && deg) {
+                const unsigned st = s_scan[tid];
+                if (st > wbase && st < wbase + Ew) s_owner[st - wbase] = (unsigned short)tid;
             }
-            DistT cur[EPT];
-#pragma unroll
-            for (int j = 0; j < EPT; ++j) {
-                const unsigned e = base + j * BT + tid;
-                nd[j] = (unsigned long long)s_d[own[j]] + a[j].y;
-                cur[j] = (e < E && nd[j] < kInf) ? ld_keep(p.dist + a[j].x, pol_keep) : (DistT)0;
-            }
-#pragma unroll
-            for (int j = 0; j < EPT; ++j) {
-                const unsigned e = base + j * BT + tid;
-                push[j] = false;
-                if (e < E) {
-                    if (nd[j] >= kInf) {
-                        atomicOr(&p.ctl->status, kStDistOverflow);  // 32-bit distances insufficient
-                    } else if (nd[j] < (unsigned long long)cur[j]) {
-                        const DistT old = atomic_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
-                        push[j] = nd[j] < (unsigned long long)old;
-                    }
+            if (tid == 0) {  // owner of the window's first arc: largest i with scan[i] <= wbase
+                unsigned lo = 0, hi = got - 1;
+                while (lo < hi) {
+                    const unsigned mid = (lo + hi + 1) >> 1;
+                    if (s_scan[mid] <= wbase) lo = mid;
+                    else hi = mid - 1;
                 }
-            }
-#pragma unroll
-            for (int j = 0; j < EPT; ++j) {
-                const unsigned o = push[j] ? adds_bucket_offset(nd[j], k, hd.h, p.nb) : 0u;
-                // head-bucket children stay in this CTA (warp-aggregated slot grab)
-                bool kept = false;
-                if (local_max) {
-                    const unsigned lm = __ballot_sync(FULL, push[j] && o == 0);
-                    if (lm) {
-                        const int leader = __ffs(lm) - 1;
-                        unsigned pos = 0;
-                        if (lane == leader) pos = atomicAdd(&s_lnext, (unsigned)__popc(lm));
-                        pos = __shfl_sync(FULL, pos, leader) + __popc(lm & lanemask_lt());
-                        if (push[j] && o == 0 && pos < local_max) {
-                            // prefetch the child's row now: its latency overlaps the rest
-                            // of this round instead of the next batch's critical path
-                            const unsigned long long rb = ld_stream_u64(p.off + a[j].x, pol_stream);
-                            const unsigned long long re = ld_stream_u64(p.off + a[j].x + 1, pol_stream);
-                            s_lv[pos] = a[j].x;
-                            s_ld[pos] = (DistT)nd[j];
-                            s_lbeg[pos] = rb;
-                            s_ldeg[pos] = (unsigned)(re - rb);
-                            kept = true;
-                        }
-                    }
-                }
-                const bool pg = push[j] && !kept;
-                const unsigned act = __ballot_sync(FULL, pg);
-                if (pg) {  // warp-aggregated staging for the ring
-                    const int leader = __ffs(act) - 1;
-                    unsigned pos = 0;
-                    if (lane == leader) pos = atomicAdd(&s_total, (unsigned)__popc(act));
-                    pos = __shfl_sync(act, pos, leader) + __popc(act & lanemask_lt());
-                    const unsigned peers = __match_any_sync(act, o);
-                    const int pl = __ffs(peers) - 1;
-                    unsigned r0 = 0;
-                    if (lane == pl) r0 = atomicAdd(&s_cnt[o], (unsigned)__popc(peers));
-                    r0 = __shfl_sync(peers, r0, pl) + __popc(peers & lanemask_lt());
-                    s_items[pos] = IT::make(a[j].x, nd[j]);
-                    s_soff[pos] = (unsigned char)o;
-                    s_rank[pos] = (unsigned short)r0;
-                }
+                s_owner[0] = (unsigned short)lo;
             }
             __syncthreads();
-            const unsigned total = s_total;
-            if (prof) s_prof[PR_N_ROUND] += 1;
-            if (total > (unsigned)(kStage - kRound) || (base + kRound >= E && total > 0)) {
-                // ---------------------------------------------------- flush to the ring
-                const long long tf = prof ? clock64() : 0;
-                if (warp == 0 && lane < (int)p.nb) {
-                    const unsigned c = s_cnt[lane];
-                    if (c) {
-                        const unsigned sl = (hs + lane) & nbm;
-                        // returning atomic: the reserve (which also counts the children for
-                        // termination) is performed before this CTA's completion atomic
-                        const unsigned long long b = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
-                        s_base[lane] = b;
-                        if (b + c > p.cap) {  // lapping: previous occupants must be claimed
-                            const unsigned long long cl = ld_relaxed_u64(&p.bk[sl].claim.v);
-                            if (b + c - p.cap > cl) atomicOr(&p.ctl->status, kStRingOverflow);
+            {
+                unsigned short* ow = s_owner + tid * kPer;
+                unsigned run[kPer];
+                unsigned m = 0;
+#pragma unroll
+                for (int i = 0; i < kPer; ++i) {
+                    m = ow[i] > m ? ow[i] : m;
+                    run[i] = m;
+                }
+                unsigned inc = m;  // warp inclusive max-scan of per-thread maxima
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const unsigned y = __shfl_up_sync(FULL, inc, o);
+                    if (lane >= o) inc = y > inc ? y : inc;
+                }
+                unsigned excl = __shfl_up_sync(FULL, inc, 1);
+                if (lane == 0) excl = 0;
+                if (lane == 31) s_wsum[warp] = inc;
+                __syncthreads();
+                unsigned wpre = 0;
+#pragma unroll
+                for (int w2 = 0; w2 < kWarps; ++w2)
+                    if (w2 < warp) wpre = s_wsum[w2] > wpre ? s_wsum[w2] : wpre;
+                const unsigned carry = excl > wpre ? excl : wpre;
+#pragma unroll
+                for (int i = 0; i < kPer; ++i) ow[i] = (unsigned short)(run[i] > carry ? run[i] : carry);
+            }
+            __syncthreads();
+            // ------------------------------------------------ async arc prefetch: the
+            // whole window in flight at once (LDGSTS), coalesced along each row
+            for (unsigned q = tid; q < Ew; q += BT) {
+                const unsigned o = s_owner[q];
+                cp_async_8(s_arc_addr + q * 8u, p.adj + s_ebeg[o] + (wbase + q - s_scan[o]), pol_stream);
+            }
+            cp_async_wait_all();
+            __syncthreads();
+            if (prof) {
+                tw += clock64() - tw0;
+                s_prof[PR_N_WINDOW] += 1;
+            }
+
+            // ------------------------------------------------ relax + push (rounds)
+            for (unsigned rbase = 0; rbase < Ew; rbase += kRound) {
+                uint2 a[EPT];
+                unsigned long long nd[EPT];
+                bool push[EPT];
+                DistT cur[EPT];
+#pragma unroll
+                for (int j = 0; j < EPT; ++j) {
+                    const unsigned q = rbase + j * BT + tid;
+                    if (q < Ew) {
+                        a[j] = s_arc[q];
+                        nd[j] = (unsigned long long)s_d[s_owner[q]] + a[j].y;
+                    } else {
+                        a[j] = make_uint2(0u, 0u);
+                        nd[j] = kInf;
+                    }
+                }
+#pragma unroll
+                for (int j = 0; j < EPT; ++j)  // EPT independent L2 gathers in flight
+                    cur[j] = nd[j] < kInf ? ld_keep(p.dist + a[j].x, pol_keep) : (DistT)0;
+#pragma unroll
+                for (int j = 0; j < EPT; ++j) {
+                    const unsigned q = rbase + j * BT + tid;
+                    push[j] = false;
+                    if (q < Ew) {
+                        if (nd[j] >= kInf) {
+                            atomicOr(&p.ctl->status, kStDistOverflow);  // 32-bit distances insufficient
+                        } else if (nd[j] < (unsigned long long)cur[j]) {
+                            const DistT old = atomic_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
+                            push[j] = nd[j] < (unsigned long long)old;
                         }
                     }
                 }
-                __syncthreads();
-                for (unsigned i = tid; i < total; i += BT) {
-                    const unsigned o = s_soff[i];
-                    const unsigned sl = (hs + o) & nbm;
-                    const unsigned long long idx = s_base[o] + s_rank[i];
-                    char* sp = p.ring + ((size_t)sl * p.cap + (idx & (p.cap - 1))) * IT::kBytes;
-                    bool ok = true;
-                    if (idx >= p.cap) {  // wait for the previous lap's reader to clear it
-                        unsigned spins = 0;
-                        while (!IT::empty(sp)) {
-                            if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) {
-                                ok = false;
-                                break;
+#pragma unroll
+                for (int j = 0; j < EPT; ++j) {
+                    if (!__any_sync(FULL, push[j])) continue;
+                    const unsigned o = push[j] ? adds_bucket_offset(nd[j], k, hd.h, p.nb) : 0u;
+                    // head-bucket children stay in this CTA (warp-aggregated slot grab)
+                    bool kept = false;
+                    if (local_max) {
+                        const unsigned lm = __ballot_sync(FULL, push[j] && o == 0);
+                        if (lm) {
+                            const int leader = __ffs(lm) - 1;
+                            unsigned pos = 0;
+                            if (lane == leader) pos = atomicAdd(&s_lnext, (unsigned)__popc(lm));
+                            pos = __shfl_sync(FULL, pos, leader) + __popc(lm & lt_mask);
+                            if (push[j] && o == 0 && pos < local_max) {
+                                s_lv[pos] = a[j].x;
+                                s_ld[pos] = (DistT)nd[j];
+                                kept = true;
                             }
                         }
                     }
-                    if (ok) IT::store(sp, s_items[i]);
-                }
-                __syncthreads();
-                if (warp == 0 && lane < (int)p.nb) {
-                    const unsigned c = s_cnt[lane];
-                    if (c) {
-                        atomicAdd(&p.bk[(hs + lane) & nbm].avail.v, (unsigned long long)c);  // publish
-                        s_cnt[lane] = 0;
+                    const bool pg = push[j] && !kept;
+                    const unsigned act = __ballot_sync(FULL, pg);
+                    if (pg) {  // warp-aggregated staging for the ring
+                        const int leader = __ffs(act) - 1;
+                        unsigned pos = 0;
+                        if (lane == leader) pos = atomicAdd(&s_total, (unsigned)__popc(act));
+                        pos = __shfl_sync(act, pos, leader) + __popc(act & lt_mask);
+                        const unsigned peers = __match_any_sync(act, o);
+                        const int pl = __ffs(peers) - 1;
+                        unsigned r0 = 0;
+                        if (lane == pl) r0 = atomicAdd(&s_cnt[o], (unsigned)__popc(peers));
+                        r0 = __shfl_sync(peers, r0, pl) + __popc(peers & lt_mask);
+                        s_items[pos] = IT::make(a[j].x, nd[j]);
+                        s_soff[pos] = (unsigned char)o;
+                        s_rank[pos] = (unsigned short)r0;
                     }
                 }
-                if (tid == 0) {
-                    s_total = 0;
-                    c_push += total;
-                }
                 __syncthreads();
-                if (prof) {
-                    tq += clock64() - tf;
-                    s_prof[PR_N_FLUSH] += 1;
+                const unsigned total = s_total;
+                if (prof) s_prof[PR_N_ROUND] += 1;
+                const bool last = (wbase + rbase + kRound >= E);
+                if (total > (unsigned)(kStage - kRound) || (last && total > 0)) {
+                    // ------------------------------------------------ flush to the ring
+                    const long long tf = prof ? clock64() : 0;
+                    if (warp == 0 && lane < (int)p.nb) {
+                        const unsigned c = s_cnt[lane];
+                        if (c) {
+                            const unsigned sl = (hs + lane) & nbm;
+                            // returning atomic: the reserve (which also counts the children for
+                            // termination) is performed before this CTA's completion atomic
+                            const unsigned long long b = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
+                            s_base[lane] = b;
+                            if (b + c > p.cap) {  // lapping: previous occupants must be claimed
+                                const unsigned long long cl = ld_relaxed_u64(&p.bk[sl].claim.v);
+                                if (b + c - p.cap > cl) atomicOr(&p.ctl->status, kStRingOverflow);
+                            }
+                        }
+                    }
+                    __syncthreads();
+                    for (unsigned i = tid; i < total; i += BT) {
+                        const unsigned o = s_soff[i];
+                        const unsigned sl = (hs + o) & nbm;
+                        const unsigned long long idx = s_base[o] + s_rank[i];
+                        char* sp = p.ring + ((size_t)sl * p.cap + (idx & (p.cap - 1))) * IT::kBytes;
+                        bool ok = true;
+                        if (idx >= p.cap) {  // wait for the previous lap's reader to clear it
+                            unsigned spins = 0;
+                            while (!IT::empty(sp)) {
+                                if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) {
+                                    ok = false;
+                                    break;
+                                }
+                            }
+                        }
+                        if (ok) IT::store(sp, s_items[i]);
+                    }
+                    __syncthreads();
+                    if (warp == 0 && lane < (int)p.nb) {
+                        const unsigned c = s_cnt[lane];
+                        if (c) {
+                            atomicAdd(&p.bk[(hs + lane) & nbm].avail.v, (unsigned long long)c);  // publish
+                            s_cnt[lane] = 0;
+                        }
+                    }
+                    if (tid == 0) {
+                        s_total = 0;
+                        c_push += total;
+                    }
+                    __syncthreads();
+                    if (prof) {
+                        tq += clock64() - tf;
+                        s_prof[PR_N_FLUSH] += 1;
+                    }
                 }
             }
         }
         if (prof) {
             const long long t1 = clock64();
-            s_prof[PR_ROUNDS] += t1 - t0 - tq;
+            s_prof[PR_ROUNDS] += t1 - t0 - tq - tw;
             s_prof[PR_FLUSH] += tq;
+            s_prof[PR_WINDOW] += tw;
             t0 = t1;
         }
 
         // ------------------------------------------------------------ complete
+        __syncthreads();  // s_lnext final (also covers the E == 0 case)
         const unsigned kept = s_lnext < local_max ? s_lnext : local_max;
         if (tid == 0) {
             // one atomic: the kept children inherit the parents' accounting
@@ -540,9 +692,22 @@ __global__ void __launch_bounds__(BT) adds_persistent_kernel(const Params<DistT>
             else if (kept > got) atomicAdd(&p.bk[slot].local.v, (unsigned long long)(kept - got));
             c_push += kept;
             c_local += kept;
+            if (kept) s_slot = slot;
+        }
+        if (p.dynamic && warp == 0) {
+            unsigned run_ctl = 0;
+            if (lane == 0) {
+                if (nlive) {
+                    atomicAdd(&p.ctl->g_exp, (unsigned long long)nlive);
+                    atomicAdd(&p.ctl->g_first, (unsigned long long)nfirst);
+                }
+                const unsigned long long now = globaltimer();
+                const unsigned long long last = ld_relaxed_u64(&p.ctl->last_ctl_ns);
+                if (now - last > p.period_ns && atomicCAS(&p.ctl->last_ctl_ns, last, now) == last) run_ctl = 1;
+            }
+            if (__shfl_sync(FULL, run_ctl, 0)) periodic_step<DistT>(p, lane);
         }
         have_local = kept;
-        if (kept) s_slot = slot;  // (uniform value; every thread writes the same)
         __syncthreads();
         if (prof) s_prof[PR_COMPLETE] += clock64() - t0;
     }

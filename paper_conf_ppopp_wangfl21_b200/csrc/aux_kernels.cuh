@@ -42,11 +42,14 @@ __global__ void interleave_kernel(const unsigned* __restrict__ col, const unsign
 
 template <typename DistT>
 __global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned source, Ctl* ctl, BucketCtl* bk,
-                                char* ring, unsigned long long cap, Head h0) {
+                                char* ring, unsigned long long cap, Head h0, unsigned* expanded) {
     using IT = ItemT<DistT>;
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
     for (unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
         dist[v] = (v == source) ? (DistT)0 : DistInf<DistT>::value;
+    const unsigned long long nw = ((unsigned long long)n + 31) / 32;
+    for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += stride)
+        expanded[i] = 0u;
     if (blockIdx.x == 0) {
         const unsigned t = threadIdx.x;
         if (t < kMaxBuckets) {
@@ -68,6 +71,8 @@ __global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned s
             ctl->head_switches = 0;
             ctl->delta_changes = 0;
             ctl->t_start = globaltimer();
+            ctl->g_exp = ctl->g_first = ctl->exp_mark = ctl->first_mark = ctl->ctl_steps = 0;
+            ctl->last_ctl_ns = ctl->t_start;
             ctl->st_vertices = ctl->st_edges = ctl->st_pushes = ctl->st_stale = ctl->st_local = 0;
             ctl->reach_v = ctl->reach_e = ctl->max_dist = 0;
             for (int i = 0; i < (int)kProfCounters; ++i) ctl->prof[i] = 0;

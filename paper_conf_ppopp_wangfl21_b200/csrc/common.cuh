@@ -26,7 +26,8 @@ constexpr unsigned kStBug = 8u;            // internal invariant violated
 // Phase profile (SSSP_FLAG_PROFILE), summed over CTAs; see sssp_get_profile().
 enum ProfIdx {
     PR_CLAIM = 0, PR_IDLE, PR_POP, PR_SCAN, PR_ROUNDS, PR_FLUSH, PR_COMPLETE, PR_TOTAL,
-    PR_N_RING, PR_N_LOCAL, PR_N_IDLE, PR_N_FLUSH, PR_N_ROUND, PR_N_CTAS, kProfCounters = 16
+    PR_N_RING, PR_N_LOCAL, PR_N_IDLE, PR_N_FLUSH, PR_N_ROUND, PR_N_CTAS, PR_WINDOW, PR_N_WINDOW,
+    kProfCounters = 16
 };
 
 struct alignas(128) Counter {
@@ -71,6 +72,7 @@ __host__ __device__ __forceinline__ unsigned meta_since(unsigned long long m) { 
 struct TraceEntry {  // mirrors sssp_trace_entry
     unsigned long long time_ns, head, pending_total, pending_window, pending_tail;
     unsigned delta_log2, active;
+    unsigned waste_permille, reason;  // reason: 1 head switch, 2 periodic step
 };
 
 struct alignas(128) Ctl {
@@ -82,6 +84,14 @@ struct alignas(128) Ctl {
     unsigned delta_changes;
     unsigned long long t_start;  // %globaltimer at init (watchdog)
     char pad2_[104];
+    // Delta-controller work signal (own lines: updated with REDs once per batch)
+    unsigned long long g_exp;     // items expanded (not stale)
+    char pad4_[120];
+    unsigned long long g_first;   // first expansions of a vertex (distinct vertices expanded)
+    char pad5_[120];
+    unsigned long long last_ctl_ns, exp_mark, first_mark;  // controller period / window start
+    unsigned long long ctl_steps;
+    char pad6_[96];
     unsigned long long st_local;  // items continued CTA-locally
     // statistics (flushed once per CTA at exit, or by finalize)
     unsigned long long st_vertices, st_edges, st_pushes, st_stale;
@@ -134,9 +144,12 @@ __device__ __forceinline__ unsigned long long policy_evict_first() {
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
     return p;
 }
-__device__ __forceinline__ unsigned long long policy_evict_last() {
+// evict_last residency is bounded by the L2 persisting set-aside
+// (cudaLimitPersistingL2CacheSize); `frac` = set-aside / dist bytes keeps a
+// stable subset of dist resident when it does not fit entirely.
+__device__ __forceinline__ unsigned long long policy_evict_last(float frac) {
     unsigned long long p;
-    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    asm volatile("createpolicy.fractional.L2::evict_last.L2::evict_unchanged.b64 %0, %1;" : "=l"(p) : "f"(frac));
     return p;
 }
 __device__ __forceinline__ uint2 ld_stream_u2(const uint2* a, unsigned long long pol) {
@@ -200,6 +213,15 @@ __device__ __forceinline__ Head ld_head(const Head* p) {
     ld_relaxed_v2u64(p, h.h, h.meta);
     return h;
 }
+
+// 8-byte asynchronous global->shared copy (LDGSTS), streamed through L2 (evict_first).
+// `sdst` is a shared-window address (convert the base once with smem_addr()).
+__device__ __forceinline__ unsigned smem_addr(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void cp_async_8(unsigned sdst, const void* gsrc, unsigned long long pol) {
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 8, %2;" ::"r"(sdst), "l"(gsrc), "l"(pol)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
 __device__ __forceinline__ unsigned lanemask_lt() {
     unsigned m;

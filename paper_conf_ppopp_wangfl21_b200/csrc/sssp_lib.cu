@@ -79,12 +79,13 @@ struct sssp_graph {
     DevBuf ring;        // nb * cap * item bytes
     unsigned long long cap = 0;
     int ring_item_bytes = 0;
-    DevBuf bk, ctl, trace, scratch, hostout;
+    DevBuf bk, ctl, trace, scratch, hostout, expanded;
     unsigned trace_alloc = 0;
     Ctl* h_ctl = nullptr;  // pinned
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
 
     int cur_bits = 32;  // 64 after a 32-bit overflow was observed (sticky)
+    size_t persist_max = 0;  // device's L2 persisting set-aside limit (bytes)
     bool busy = false;
     bool async_pending = false;
     sssp_stats stats{};
@@ -114,29 +115,32 @@ sssp_status check_options(const sssp_options& o) {
         return fail(SSSP_ERR_INVALID_ARGUMENT, "block_threads must be 0, 128, 256 or 512");
     if (o.clip_pct == 0 || o.clip_pct > 100) return fail(SSSP_ERR_INVALID_ARGUMENT, "clip_pct");
     if (o.active_init > o.num_buckets) return fail(SSSP_ERR_INVALID_ARGUMENT, "active_init > num_buckets");
+    if (o.waste_lo_permille > 1000 || o.waste_hi_permille > 1000) return fail(SSSP_ERR_INVALID_ARGUMENT, "waste permille");
     return SSSP_OK;
 }
 
 // ----------------------------------------------------------------- kernel table
-// arcs per thread per round: 4 keeps 4 independent 8-byte loads in flight per
-// thread; halved where the staging buffer would exceed 48 KB of static smem
+// Kernel variants: <dist type, CTA size, arcs per thread per round (EPT),
+// arc-window size W>.  EPT = 4 independent L2 gathers in flight per thread;
+// W = 2048 arcs (16 KB) prefetched asynchronously per window.
+struct KVariant {
+    void* fn;
+    size_t smem;
+};
 template <typename DistT, int BT>
-constexpr int ept() {
-    return (sizeof(DistT) == 8 && BT >= 512) ? 1 : (sizeof(DistT) == 8 || BT >= 512) ? 2 : 4;
+KVariant kvar() {
+    constexpr int W = BT >= 256 ? 2048 : 1024;
+    return KVariant{(void*)adds_persistent_kernel<DistT, BT, 4, W>, Smem<DistT, BT, 4, W>::bytes};
 }
-template <typename DistT, int BT>
-void* kfun() {
-    return (void*)adds_persistent_kernel<DistT, BT, ept<DistT, BT>()>;
-}
-void* persistent_fn(int bits, int bt) {
+KVariant persistent_variant(int bits, int bt) {
     if (bits == 32) {
-        if (bt == 128) return kfun<uint32_t, 128>();
-        if (bt == 512) return kfun<uint32_t, 512>();
-        return kfun<uint32_t, 256>();
+        if (bt == 128) return kvar<uint32_t, 128>();
+        if (bt == 512) return kvar<uint32_t, 512>();
+        return kvar<uint32_t, 256>();
     }
-    if (bt == 128) return kfun<unsigned long long, 128>();
-    if (bt == 512) return kfun<unsigned long long, 512>();
-    return kfun<unsigned long long, 256>();
+    if (bt == 128) return kvar<unsigned long long, 128>();
+    if (bt == 512) return kvar<unsigned long long, 512>();
+    return kvar<unsigned long long, 256>();
 }
 
 sssp_status ensure_ring(sssp_graph* g, int item_bytes, unsigned long long cap) {
@@ -196,6 +200,22 @@ Params<DistT> make_params(sssp_graph* g, unsigned grid, unsigned bt, unsigned k_
     p.local_max = (g->opts.flags & SSSP_FLAG_NO_LOCAL) ? 0u : (g->opts.local_max ? g->opts.local_max : bt);
     p.max_backoff_ns = g->opts.max_backoff_ns ? g->opts.max_backoff_ns : 2048u;
     p.prof = (g->opts.flags & SSSP_FLAG_PROFILE) ? 1u : 0u;
+    // L2 residency of dist (D5): reserve the persisting set-aside for
+    // it and mark dist accesses evict_last over the fraction that fits
+    p.expanded = (unsigned*)g->expanded.p;
+    p.waste_lo = g->opts.waste_lo_permille;
+    p.waste_hi = g->opts.waste_hi_permille;
+    p.period_ns = (unsigned long long)(g->opts.period_us ? g->opts.period_us : 20u) * 1000ull;
+    p.keep_frac = 0.0f;
+    if (!(g->opts.flags & SSSP_FLAG_NO_L2_PERSIST) && g->persist_max) {
+        const size_t want = (size_t)g->n * sizeof(DistT);
+        const size_t use = std::min(want, g->persist_max);
+        size_t cur = 0;
+        cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+        if (cur < use) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, use);
+        cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+        p.keep_frac = want ? (float)std::min(1.0, (double)std::min(cur, use) / (double)want) : 0.0f;
+    }
     p.k_max = k_max;
     p.timeout_ns = (unsigned long long)(g->opts.timeout_ms ? g->opts.timeout_ms : 60000u) * 1000000ull;
     return p;
@@ -206,9 +226,11 @@ template <typename DistT>
 sssp_status launch_one(sssp_graph* g, uint32_t source, unsigned long long* out_dev, cudaStream_t s, int bits,
                        unsigned k0) {
     const unsigned bt = g->opts.block_threads ? g->opts.block_threads : 256;
-    void* fn = persistent_fn(bits, (int)bt);
+    const KVariant kv = persistent_variant(bits, (int)bt);
+    void* fn = kv.fn;
+    CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kv.smem), "smem attribute");
     int occ = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, (int)bt, 0), "occupancy query");
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, (int)bt, kv.smem), "occupancy query");
     if (occ < 1) return fail(SSSP_ERR_CUDA, "persistent kernel cannot be resident");
     unsigned grid = (unsigned)(occ * g->sm_count);
     if (g->opts.grid_ctas && g->opts.grid_ctas < grid) grid = g->opts.grid_ctas;
@@ -220,11 +242,12 @@ sssp_status launch_one(sssp_graph* g, uint32_t source, unsigned long long* out_d
 
     const unsigned aux_grid = (unsigned)g->sm_count * 8;
     CK(cudaEventRecord(g->ev[0], s), "event");
-    init_run_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, g->n, source, p.ctl, p.bk, p.ring, g->cap, h0);
+    init_run_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, g->n, source, p.ctl, p.bk, p.ring, g->cap, h0,
+                                                    p.expanded);
     CK(cudaGetLastError(), "init kernel launch");
     CK(cudaEventRecord(g->ev[1], s), "event");
     void* args[] = {(void*)&p};
-    CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(bt), args, 0, s), "persistent kernel launch");
+    CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(bt), args, kv.smem, s), "persistent kernel launch");
     CK(cudaEventRecord(g->ev[2], s), "event");
     finalize_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, out_dev, g->n, g->d_off, p.ctl);
     CK(cudaGetLastError(), "finalize kernel launch");
@@ -390,6 +413,9 @@ void sssp_options_default(sssp_options* o) {
     o->settle_head_switches = 2;   // P:215 (reading R7)
     o->util_lo_pct = 100;          // P:211 (reading R6)
     o->util_hi_pct = 400;
+    o->waste_lo_permille = 200;    // reading R6: grow Delta only while < 20% of expansions are repeats
+    o->waste_hi_permille = 450;    //             shrink it while > 45% are (work <~ 1.8x Dijkstra)
+    o->period_us = 20;
     o->dist_bits = 0;
     o->ring_items = 0;
     o->flags = 0;
@@ -429,6 +455,7 @@ sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offset
     g->m = m;
     g->opts = o;
     g->sm_count = prop.multiProcessorCount;
+    g->persist_max = prop.persistingL2CacheMaxSize > 0 ? (size_t)prop.persistingL2CacheMaxSize : 0;
     auto bail = [&](sssp_status s2) {
         sssp_graph_destroy(g);
         return s2;
@@ -494,6 +521,7 @@ sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offset
 
     CKG(cudaMalloc(&g->dist.p, (size_t)n * 8), "allocating dist");
     g->dist.bytes = (size_t)n * 8;
+    CKG(cudaMalloc(&g->expanded.p, ((size_t)n + 31) / 32 * 4), "allocating the expansion bitmap");
     CKG(cudaMalloc(&g->bk.p, sizeof(BucketCtl) * kMaxBuckets), "allocating bucket counters");
     CKG(cudaMemset(g->bk.p, 0, sizeof(BucketCtl) * kMaxBuckets), "bucket counters");
     CKG(cudaMalloc(&g->ctl.p, sizeof(Ctl)), "allocating control block");
@@ -519,6 +547,7 @@ sssp_status sssp_graph_destroy(sssp_graph* g) {
     g->ctl.release();
     g->trace.release();
     g->scratch.release();
+    g->expanded.release();
     g->hostout.release();
     if (g->h_ctl) cudaFreeHost(g->h_ctl);
     for (auto& e : g->ev)
