@@ -86,13 +86,14 @@ typedef struct sssp_options {
     uint64_t delta_init;       /* initial Delta; 0 = heuristic C*W/D rounded
                                   to the nearest power of two; else rounded to a power of two */
     uint32_t clip_pct;         /* tail-bucket share that raises Delta and its floor; default 65 */
-    uint32_t settle_head_switches; /* K head-bucket switches between Delta changes; default 2 */
+    uint32_t settle_head_switches; /* K controller steps (head switches or periodic steps) between Delta
+                                      changes; default 8 */
     uint32_t util_lo_pct;      /* lower utilisation limit, % of resident threads; default 100 */
     uint32_t util_hi_pct;      /* upper utilisation limit, % of resident threads; default 400 */
     uint32_t waste_lo_permille;/* Delta may grow only while the recent re-expansion share is below this
-                                  (default 200 = 20%) */
+                                  (default 50 = 5%) */
     uint32_t waste_hi_permille;/* Delta shrinks (not below its clip floor) while the share is above this
-                                  (default 450 = 45%, i.e. ~1.8x Dijkstra's vertex work) */
+                                  (default 500 = 50%, i.e. ~2x Dijkstra's vertex work) */
     uint32_t period_us;        /* periodic controller step (default 20 us; head switches also step) */
     uint32_t dist_bits;        /* 0 = auto (32-bit internal distances when provably or observably
                                   safe, else 64), 32 or 64 */

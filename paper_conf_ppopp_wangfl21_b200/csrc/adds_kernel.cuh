@@ -89,7 +89,8 @@ __device__ __forceinline__ long long warp_sum_s64(long long x) {
 // window (utilisation = window items x average degree vs resident threads,
 // P:211) and the tail (clip share); plus the recent re-expansion
 // share of expansions (work-waste signal, R6).  Readings:
-//   clip   tail >= clip_pct of all pending        -> Delta x2, floor = Delta
+//   clip   tail >= clip_pct of all pending, or >= 1/4 of recent pushes were
+//          clipped into the tail                  -> Delta x2, floor = Delta
 //   waste  share > waste_hi after settling        -> Delta /2 (not below floor)
 //   grow   window under-utilised AND share < lo   -> Delta x2
 //   A      active buckets follow the same two signals one step at a time
@@ -102,7 +103,8 @@ struct CtlDecision {
 
 template <typename DistT>
 __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, unsigned flo, unsigned since,
-                              long long total, long long tail, long long win, unsigned waste, bool waste_known) {
+                              long long total, long long tail, long long win, unsigned waste, bool waste_known,
+                              unsigned clip, bool clip_known) {
     CtlDecision d{k, A, flo, since + 1, false};
     if (!p.dynamic) return d;
     const unsigned long long util = ((unsigned long long)(win > 0 ? win : 0) * p.avg_deg_x16) >> 4;
@@ -111,7 +113,8 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
     const bool high = util * 100ull > (unsigned long long)p.util_hi_pct * T;
     const bool wasteful = waste_known && waste > p.waste_hi;
     const bool frugal = waste_known && waste < p.waste_lo;
-    if (total >= 64 && tail * 100 >= (long long)p.clip_pct * total && k < p.k_max) {
+    const bool clipping = (total >= 64 && tail * 100 >= (long long)p.clip_pct * total) || (clip_known && clip >= 250);
+    if (clipping && k < p.k_max) {
         d.k = k + 1;  // clipping: raise Delta and its lower bound
         d.flo = d.k;
         d.changed = true;
@@ -152,6 +155,13 @@ __device__ __forceinline__ unsigned recent_waste(const Params<DistT>& p, bool& k
     known = e >= 4096;
     return (known && e > f) ? (unsigned)((e - f) * 1000ull / e) : 0u;
 }
+template <typename DistT>
+__device__ __forceinline__ unsigned recent_clip(const Params<DistT>& p, bool& known) {
+    const unsigned long long q = ld_relaxed_u64(&p.ctl->g_push) - ld_relaxed_u64(&p.ctl->push_mark);
+    const unsigned long long c = ld_relaxed_u64(&p.ctl->g_clip) - ld_relaxed_u64(&p.ctl->clip_mark);
+    known = q >= 1024;
+    return known ? (unsigned)(c * 1000ull / q) : 0u;
+}
 
 // Commit a controller step by 128-bit CAS; restart the waste window on a change
 // (and every 8 steps so the signal tracks the recent past).
@@ -165,6 +175,8 @@ __device__ void commit_step(const Params<DistT>& p, const Head hd, const Head nh
     if (kchanged || (since & 7) == 0) {
         p.ctl->exp_mark = ld_relaxed_u64(&p.ctl->g_exp);
         p.ctl->first_mark = ld_relaxed_u64(&p.ctl->g_first);
+        p.ctl->push_mark = ld_relaxed_u64(&p.ctl->g_push);
+        p.ctl->clip_mark = ld_relaxed_u64(&p.ctl->g_clip);
     }
     if (p.trace_cap) {
         const unsigned t = atomicAdd(&p.ctl->trace_count, 1u);
@@ -215,9 +227,11 @@ __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lan
     const long long tail = __shfl_sync(FULL, pend, nb - 1);
     const long long win = warp_sum_s64((lane >= (int)o && lane < (int)(o + A)) ? pend : 0);
     if (lane != 0) return false;
-    bool known;
+    bool known, cknown;
     const unsigned waste = recent_waste(p, known);
-    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), total, tail, win, waste, known);
+    const unsigned clip = recent_clip(p, cknown);
+    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), total, tail, win, waste, known,
+                                 clip, cknown);
     const Head nhd{rehead(hd.h + o, k, d.k),
                    pack_meta((hs + o) & (nb - 1), d.k, d.A, d.flo, d.since > 0xffff ? 0xffff : d.since)};
     commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 1u);
@@ -236,9 +250,11 @@ __device__ void periodic_step(const Params<DistT>& p, const int lane) {
     const long long tail = __shfl_sync(FULL, pend, p.nb - 1);
     const long long win = warp_sum_s64(lane < (int)A ? pend : 0);
     if (lane != 0 || total == 0) return;
-    bool known;
+    bool known, cknown;
     const unsigned waste = recent_waste(p, known);
-    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), total, tail, win, waste, known);
+    const unsigned clip = recent_clip(p, cknown);
+    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), total, tail, win, waste, known,
+                                 clip, cknown);
     const Head nhd{rehead(hd.h, k, d.k), pack_meta(hs, d.k, d.A, d.flo, d.since > 0xffff ? 0xffff : d.since)};
     commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 2u);
 }
@@ -625,6 +641,10 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                     const long long tf = prof ? clock64() : 0;
                     if (warp == 0 && lane < (int)p.nb) {
                         const unsigned c = s_cnt[lane];
+                        if (p.dynamic) {
+                            if (lane == 0) atomicAdd(&p.ctl->g_push, (unsigned long long)total);
+                            if (lane == (int)nbm && c) atomicAdd(&p.ctl->g_clip, (unsigned long long)c);
+                        }
                         if (c) {
                             const unsigned sl = (hs + lane) & nbm;
                             // returning atomic: the reserve (which also counts the children for
@@ -701,6 +721,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                     atomicAdd(&p.ctl->g_exp, (unsigned long long)nlive);
                     atomicAdd(&p.ctl->g_first, (unsigned long long)nfirst);
                 }
+                if (kept) atomicAdd(&p.ctl->g_push, (unsigned long long)kept);
                 const unsigned long long now = globaltimer();
                 const unsigned long long last = ld_relaxed_u64(&p.ctl->last_ctl_ns);
                 if (now - last > p.period_ns && atomicCAS(&p.ctl->last_ctl_ns, last, now) == last) run_ctl = 1;

@@ -90,8 +90,12 @@ struct alignas(128) Ctl {
     unsigned long long g_first;   // first expansions of a vertex (distinct vertices expanded)
     char pad5_[120];
     unsigned long long last_ctl_ns, exp_mark, first_mark;  // controller period / window start
-    unsigned long long ctl_steps;
-    char pad6_[96];
+    unsigned long long push_mark, clip_mark;
+    char pad6_[88];
+    unsigned long long g_push;    // items pushed (ring + kept)
+    char pad7_[120];
+    unsigned long long g_clip;    // items pushed into the tail bucket (clipped)
+    char pad8_[120];
     unsigned long long st_local;  // items continued CTA-locally
     // statistics (flushed once per CTA at exit, or by finalize)
     unsigned long long st_vertices, st_edges, st_pushes, st_stale;

@@ -410,11 +410,11 @@ void sssp_options_default(sssp_options* o) {
     o->delta_mode = SSSP_DELTA_DYNAMIC;
     o->delta_init = 0;             // heuristic C*W/D
     o->clip_pct = 65;
-    o->settle_head_switches = 2;   // P:215 (reading R7)
+    o->settle_head_switches = 8;   // P:215 (reading R7): controller steps between Delta changes
     o->util_lo_pct = 100;          // P:211 (reading R6)
     o->util_hi_pct = 400;
-    o->waste_lo_permille = 200;    // reading R6: grow Delta only while < 20% of expansions are repeats
-    o->waste_hi_permille = 450;    //             shrink it while > 45% are (work <~ 1.8x Dijkstra)
+    o->waste_lo_permille = 50;     // reading R6: grow Delta only while < 5% of expansions are repeats
+    o->waste_hi_permille = 500;    //             shrink it while > 50% are (work <~ 2x Dijkstra)
     o->period_us = 20;
     o->dist_bits = 0;
     o->ring_items = 0;

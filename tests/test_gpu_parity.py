@@ -201,11 +201,16 @@ def test_trace_invariants():
     assert np.array_equal(d, oracle.dijkstra(g, s)[0])
     st = G.stats()
     tr = G.trace()
-    assert len(tr) == min(st["head_switches"], 65536)
+    assert sum(1 for e in tr if e["reason"] == 1) == min(st["head_switches"], 65536)
     for e in tr:
+        assert e["reason"] in (1, 2)
         assert 1 <= e["active"] <= 32
         assert 0 <= e["delta_log2"] <= 31
+        assert e["waste_permille"] <= 1000
         assert e["pending_tail"] <= e["pending_total"] and e["pending_window"] <= e["pending_total"]
+    # Delta moves one power of two per step and only after settling, except clip steps
+    ks = [e["delta_log2"] for e in tr]
+    assert all(abs(a - b) <= 1 for a, b in zip(ks, ks[1:]))
     ts = [e["time_ns"] for e in tr]
     assert len(tr) < 2 or max(ts) >= min(ts)
 
