@@ -70,9 +70,16 @@ typedef enum sssp_status {
 #define SSSP_FLAG_NO_RETRY 0x4u  /* on worklist overflow return SSSP_ERR_WORKLIST_OVERFLOW instead of growing */
 #define SSSP_FLAG_NO_LOCAL 0x8u  /* publish every child through the ring (ablation of CTA-local continuation) */
 #define SSSP_FLAG_PROFILE 0x10u  /* accumulate per-phase SM-cycle counters (sssp_get_profile) */
+#define SSSP_FLAG_ADAPT_ACTIVE 0x40u  /* let the controller vary the number of active buckets;
+                                        off by default: on our workloads it raised re-expansions */
 #define SSSP_FLAG_NO_L2_PERSIST 0x20u /* do not reserve the L2 persisting set-aside for dist (ablation).
                                         By default a run raises cudaLimitPersistingL2CacheSize (device-wide)
                                         up to min(dist bytes, device maximum) */
+
+/* Initial-Delta heuristics (options.delta_heuristic) */
+#define SSSP_DELTA_H_RING_SPAN 0u
+#define SSSP_DELTA_H_MAXW_OVER_D 2u
+#define SSSP_DELTA_H_NEARFAR 1u
 
 /* Delta modes */
 #define SSSP_DELTA_DYNAMIC 0u    /* ADDS: run-time controller */
@@ -83,24 +90,30 @@ typedef struct sssp_options {
     int32_t device;            /* CUDA device ordinal (default 0) */
     uint32_t num_buckets;      /* ring size B, power of two in [2, 32]; default 32 */
     uint32_t delta_mode;       /* SSSP_DELTA_DYNAMIC (default) or SSSP_DELTA_STATIC */
-    uint64_t delta_init;       /* initial Delta; 0 = heuristic C*W/D rounded
-                                  to the nearest power of two; else rounded to a power of two */
+    uint64_t delta_init;       /* initial Delta; 0 = heuristic (see delta_heuristic) rounded to the
+                                  nearest power of two; else rounded to a power of two */
     uint32_t clip_pct;         /* tail-bucket share that raises Delta and its floor; default 65 */
     uint32_t settle_head_switches; /* K controller steps (head switches or periodic steps) between Delta
                                       changes; default 8 */
     uint32_t util_lo_pct;      /* lower utilisation limit, % of resident threads; default 100 */
     uint32_t util_hi_pct;      /* upper utilisation limit, % of resident threads; default 400 */
     uint32_t waste_lo_permille;/* Delta may grow only while the recent re-expansion share is below this
-                                  (default 50 = 5%) */
+                                  (default 350 = 35%) */
     uint32_t waste_hi_permille;/* Delta shrinks (not below its clip floor) while the share is above this
                                   (default 500 = 50%, i.e. ~2x Dijkstra's vertex work) */
     uint32_t period_us;        /* periodic controller step (default 20 us; head switches also step) */
+    uint32_t delta_heuristic;  /* initial-Delta heuristic when delta_init == 0 ("a heuristic similar
+                                  to the one described in Section 4.3"): SSSP_DELTA_H_RING_SPAN (default:
+                                  max weight / num_buckets, so one maximum-weight hop from the head stays
+                                  inside the ring -- the clipping argument of P:195), SSSP_DELTA_H_MAXW_OVER_D
+                                  (max weight / average degree, Meyer-Sanders [15]) or SSSP_DELTA_H_NEARFAR
+                                  (C * W / D with C = 32, the Near-Far rule of P:120) */
     uint32_t dist_bits;        /* 0 = auto (32-bit internal distances when provably or observably
                                   safe, else 64), 32 or 64 */
     uint64_t ring_items;       /* capacity of each bucket's circular array (items, rounded up to a
                                   power of two, >= 64); 0 = auto = max(2^16, next_pow2(n)) */
     uint32_t flags;            /* SSSP_FLAG_* */
-    uint32_t block_threads;    /* worker CTA size: 0 = auto (256), else 128/256/512 */
+    uint32_t block_threads;    /* worker CTA size: 0 = auto (512), else 128/256/512 */
     uint32_t grid_ctas;        /* 0 = every co-resident CTA; else at most this many CTAs */
     uint32_t batch_min;        /* minimum items a CTA claims when enough are available; 0 = auto */
     uint32_t timeout_ms;       /* device watchdog (globaltimer); 0 = default 60000 */
@@ -109,7 +122,10 @@ typedef struct sssp_options {
     uint32_t local_max;        /* head-bucket children a CTA keeps as its own next batch instead of
                                   publishing them (0 = auto = block_threads; see SSSP_FLAG_NO_LOCAL) */
     uint32_t max_backoff_ns;   /* idle CTAs back off exponentially up to this (0 = auto = 2048) */
-    uint32_t reserved[3];
+    uint32_t startup_permille; /* the controller may not grow Delta before this share of the vertices
+                                  has been expanded or 256 head switches have happened (start-up
+                                  frontiers are always small); default 2 */
+    uint32_t reserved[1];
 } sssp_options;
 
 typedef struct sssp_stats {
@@ -147,7 +163,10 @@ typedef struct sssp_trace_entry {
     uint32_t delta_log2;     /* Delta in force after the step */
     uint32_t active;         /* active buckets after the step */
     uint32_t waste_permille; /* re-expansion share of recent expansions (work-waste signal) */
-    uint32_t reason;         /* 1 = head-bucket switch, 2 = periodic controller step */
+    uint32_t reason;         /* bits 0-7: 1 = head-bucket switch, 2 = periodic controller step;
+                                bits 8+: decision inputs (1 low util, 2 high util, 4 work beyond the
+                                window, 8 wasteful, 16 frugal, 32 clipping, 64 waste known,
+                                128 start-up over, 256 settled) */
 } sssp_trace_entry;
 
 /* Opaque handle: owns the device CSR, the workspace (bucket ring, counters,
@@ -210,7 +229,9 @@ sssp_status sssp_get_trace(sssp_graph *g, sssp_trace_entry *out, uint32_t cap, u
 sssp_status sssp_get_profile(sssp_graph *g, uint64_t *out, uint32_t cap, uint32_t *count);
 
 /* Graph facts: n, m, sum of weights, max weight, and the heuristic initial
- * Delta (log2) = round(log2(C * W / D)), C = 32, W = sum_w/m, D = m/n. */
+ * Delta (log2) under options.delta_heuristic: round(log2(max_w / B)),
+ * round(log2(max_w / D)) or round(log2(C * W / D)) with C = 32, W = sum_w/m,
+ * D = m/n. */
 sssp_status sssp_graph_info(const sssp_graph *g, uint32_t *n, uint64_t *m, uint64_t *sum_w,
                             uint32_t *max_w, uint32_t *heuristic_delta_log2);
 

@@ -33,9 +33,13 @@ SSSP_FLAG_NO_RETRY = 0x4
 SSSP_FLAG_NO_LOCAL = 0x8
 SSSP_FLAG_PROFILE = 0x10
 SSSP_FLAG_NO_L2_PERSIST = 0x20
+SSSP_FLAG_ADAPT_ACTIVE = 0x40
 PROFILE_FIELDS = ["cyc_claim", "cyc_idle", "cyc_pop", "cyc_scan", "cyc_rounds", "cyc_flush", "cyc_complete",
                   "cyc_total", "n_ring_batches", "n_local_batches", "n_idle", "n_flush", "n_rounds", "n_ctas",
                   "cyc_window", "n_windows"]
+SSSP_DELTA_H_RING_SPAN = 0
+SSSP_DELTA_H_NEARFAR = 1
+SSSP_DELTA_H_MAXW_OVER_D = 2
 SSSP_DELTA_DYNAMIC = 0
 SSSP_DELTA_STATIC = 1
 
@@ -60,11 +64,12 @@ class sssp_options(ctypes.Structure):
         ("settle_head_switches", ctypes.c_uint32), ("util_lo_pct", ctypes.c_uint32),
         ("util_hi_pct", ctypes.c_uint32), ("waste_lo_permille", ctypes.c_uint32),
         ("waste_hi_permille", ctypes.c_uint32), ("period_us", ctypes.c_uint32),
+        ("delta_heuristic", ctypes.c_uint32),
         ("dist_bits", ctypes.c_uint32), ("ring_items", ctypes.c_uint64),
         ("flags", ctypes.c_uint32), ("block_threads", ctypes.c_uint32), ("grid_ctas", ctypes.c_uint32),
         ("batch_min", ctypes.c_uint32), ("timeout_ms", ctypes.c_uint32), ("trace_capacity", ctypes.c_uint32),
         ("active_init", ctypes.c_uint32), ("local_max", ctypes.c_uint32), ("max_backoff_ns", ctypes.c_uint32),
-        ("reserved", ctypes.c_uint32 * 3),
+        ("startup_permille", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 1),
     ]
 
 

@@ -57,6 +57,7 @@ struct Params {
     unsigned nb;               // ring buckets, power of two <= 32
     unsigned long long cap;    // items per bucket array, power of two
     unsigned dynamic;          // Delta controller enabled
+    unsigned adapt_active;     // controller may vary the active-bucket count
     unsigned clip_pct;         // P:207 (65)
     unsigned settle;           // P:215 head switches between Delta changes
     unsigned util_lo_pct, util_hi_pct;  // P:211 limits, % of resident threads
@@ -71,6 +72,7 @@ struct Params {
     unsigned* expanded;        // n-bit bitmap: vertex expanded at least once (controller waste signal)
     unsigned waste_lo, waste_hi;  // permille
     unsigned long long period_ns;
+    unsigned long long startup_first;  // no Delta growth before this many first expansions
     unsigned k_max;
     unsigned long long timeout_ns;
 };
@@ -89,8 +91,8 @@ __device__ __forceinline__ long long warp_sum_s64(long long x) {
 // window (utilisation = window items x average degree vs resident threads,
 // P:211) and the tail (clip share); plus the recent re-expansion
 // share of expansions (work-waste signal, R6).  Readings:
-//   clip   tail >= clip_pct of all pending, or >= 1/4 of recent pushes were
-//          clipped into the tail                  -> Delta x2, floor = Delta
+//   clip   tail >= clip_pct of all pending, or >= 1/2 of recent pushes were
+//          clipped into the tail (2 steps apart)  -> Delta x2, floor = Delta
 //   waste  share > waste_hi after settling        -> Delta /2 (not below floor)
 //   grow   window under-utilised AND share < lo   -> Delta x2
 //   A      active buckets follow the same two signals one step at a time
@@ -99,22 +101,34 @@ __device__ __forceinline__ long long warp_sum_s64(long long x) {
 struct CtlDecision {
     unsigned k, A, flo, since;
     bool changed;
+    unsigned flags;  // decision inputs, recorded in the trace: 1 low, 2 high, 4 beyond, 8 wasteful,
+                     // 16 frugal, 32 clipping, 64 waste known, 128 progressed, 256 settled
 };
 
+// ratio_x100 = 100 * expansions / distinct vertices expanded so far (cumulative,
+// >= 100; 100 = Dijkstra's vertex work).  waste = re-expansion share (permille)
+// over the recent window.  clip = share of recent pushes that were clipped.
 template <typename DistT>
 __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, unsigned flo, unsigned since,
                               long long total, long long tail, long long win, unsigned waste, bool waste_known,
-                              unsigned clip, bool clip_known) {
-    CtlDecision d{k, A, flo, since + 1, false};
+                              unsigned clip, bool clip_known, unsigned ratio_x100, bool progressed) {
+    CtlDecision d{k, A, flo, since + 1, false, 0u};
     if (!p.dynamic) return d;
     const unsigned long long util = ((unsigned long long)(win > 0 ? win : 0) * p.avg_deg_x16) >> 4;
     const unsigned long long T = p.resident_threads;
     const bool low = util * 100ull < (unsigned long long)p.util_lo_pct * T;
     const bool high = util * 100ull > (unsigned long long)p.util_hi_pct * T;
-    const bool wasteful = waste_known && waste > p.waste_hi;
-    const bool frugal = waste_known && waste < p.waste_lo;
-    const bool clipping = (total >= 64 && tail * 100 >= (long long)p.clip_pct * total) || (clip_known && clip >= 250);
-    if (clipping && k < p.k_max) {
+    const bool beyond = (total - win) > win;  // more work waits outside the active window
+    // waste: recent re-expansions high AND the run as a whole already above 2x
+    const bool wasteful = waste_known && waste > p.waste_hi && ratio_x100 > 200;
+    // frugal: recent and cumulative re-expansion both low
+    // (no growth during the start-up transient: the first frontier is always small)
+    const bool frugal = waste_known && waste < p.waste_lo && ratio_x100 < 125 && progressed;
+    const bool clipping = (total >= 64 && tail * 100 >= (long long)p.clip_pct * total) || (clip_known && clip >= 500);
+    d.flags = (low ? 1u : 0u) | (high ? 2u : 0u) | (beyond ? 4u : 0u) | (wasteful ? 8u : 0u) |
+              (frugal ? 16u : 0u) | (clipping ? 32u : 0u) | (waste_known ? 64u : 0u) | (progressed ? 128u : 0u) |
+              (d.since >= p.settle ? 256u : 0u);
+    if (clipping && k < p.k_max && d.since >= 2) {
         d.k = k + 1;  // clipping: raise Delta and its lower bound
         d.flo = d.k;
         d.changed = true;
@@ -122,14 +136,22 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
         if (wasteful && k > flo) {
             d.k = k - 1;
             d.changed = true;
-        } else if (low && frugal && k < p.k_max) {
+        } else if (low && frugal && beyond && k < p.k_max) {
             d.k = k + 1;
             d.changed = true;
         }
     }
     if (d.changed) d.since = 0;
-    if (low && frugal && A < p.nb) d.A = A + 1;
-    else if ((wasteful || high) && A > 1) d.A = A - 1;
+    // fine-grained knob: one more active bucket only when the hardware is
+    // under-utilised, work waits beyond the window and almost nothing is
+    // re-expanded; back to fewer when wasteful or busy
+    if (p.adapt_active) {
+        if (low && beyond && waste_known && waste < p.waste_lo / 4 && ratio_x100 < 115 && d.since >= p.settle &&
+            A < p.nb)
+            d.A = A + 1;
+        else if ((wasteful || high) && A > 1)
+            d.A = A - 1;
+    }
     return d;
 }
 
@@ -156,26 +178,37 @@ __device__ __forceinline__ unsigned recent_waste(const Params<DistT>& p, bool& k
     return (known && e > f) ? (unsigned)((e - f) * 1000ull / e) : 0u;
 }
 template <typename DistT>
+__device__ __forceinline__ unsigned cumulative_ratio(const Params<DistT>& p) {
+    const unsigned long long e = ld_relaxed_u64(&p.ctl->g_exp), f = ld_relaxed_u64(&p.ctl->g_first);
+    return f >= 4096 ? (unsigned)(e * 100ull / f) : 100u;
+}
+template <typename DistT>
 __device__ __forceinline__ unsigned recent_clip(const Params<DistT>& p, bool& known) {
     const unsigned long long q = ld_relaxed_u64(&p.ctl->g_push) - ld_relaxed_u64(&p.ctl->push_mark);
     const unsigned long long c = ld_relaxed_u64(&p.ctl->g_clip) - ld_relaxed_u64(&p.ctl->clip_mark);
-    known = q >= 1024;
+    known = q >= 65536;  // a statistically meaningful sample of the push distribution
     return known ? (unsigned)(c * 1000ull / q) : 0u;
 }
 
-// Commit a controller step by 128-bit CAS; restart the waste window on a change
-// (and every 8 steps so the signal tracks the recent past).
+// Commit a controller step by 128-bit CAS; restart the measurement windows on a
+// change and whenever they are full, so the signals track the recent past.
 template <typename DistT>
 __device__ void commit_step(const Params<DistT>& p, const Head hd, const Head nhd, bool kchanged, unsigned since,
-                            long long total, long long win, long long tail, unsigned waste, unsigned reason) {
+                            long long total, long long win, long long tail, unsigned waste, unsigned reason,
+                            unsigned flags) {
     Head seen;
     if (!cas_head(&p.ctl->head, hd, nhd, seen)) return;
     if (reason == 1) atomicAdd(&p.ctl->head_switches, 1u);
     if (kchanged) atomicAdd(&p.ctl->delta_changes, 1u);
-    if (kchanged || (since & 7) == 0) {
-        p.ctl->exp_mark = ld_relaxed_u64(&p.ctl->g_exp);
+    // measurement windows are sized in events, not steps: restart after a Delta
+    // change, or once a window holds 64K expansions / 256K pushes
+    const unsigned long long ge = ld_relaxed_u64(&p.ctl->g_exp), gp = ld_relaxed_u64(&p.ctl->g_push);
+    if (kchanged || ge - ld_relaxed_u64(&p.ctl->exp_mark) >= 65536) {
+        p.ctl->exp_mark = ge;
         p.ctl->first_mark = ld_relaxed_u64(&p.ctl->g_first);
-        p.ctl->push_mark = ld_relaxed_u64(&p.ctl->g_push);
+    }
+    if (kchanged || gp - ld_relaxed_u64(&p.ctl->push_mark) >= 262144) {
+        p.ctl->push_mark = gp;
         p.ctl->clip_mark = ld_relaxed_u64(&p.ctl->g_clip);
     }
     if (p.trace_cap) {
@@ -190,7 +223,7 @@ __device__ void commit_step(const Params<DistT>& p, const Head hd, const Head nh
             e.delta_log2 = meta_k(nhd.meta);
             e.active = meta_A(nhd.meta);
             e.waste_permille = waste;
-            e.reason = reason;
+            e.reason = reason | (flags << 8);
             p.trace[t] = e;
         }
     }
@@ -231,10 +264,12 @@ __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lan
     const unsigned waste = recent_waste(p, known);
     const unsigned clip = recent_clip(p, cknown);
     const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), total, tail, win, waste, known,
-                                 clip, cknown);
+                                 clip, cknown, cumulative_ratio(p),
+                                 ld_relaxed_u64(&p.ctl->g_first) >= p.startup_first ||
+                                     ld_relaxed_u32(&p.ctl->head_switches) >= 256u);
     const Head nhd{rehead(hd.h + o, k, d.k),
                    pack_meta((hs + o) & (nb - 1), d.k, d.A, d.flo, d.since > 0xffff ? 0xffff : d.since)};
-    commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 1u);
+    commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 1u, d.flags);
     return false;
 }
 
@@ -254,9 +289,11 @@ __device__ void periodic_step(const Params<DistT>& p, const int lane) {
     const unsigned waste = recent_waste(p, known);
     const unsigned clip = recent_clip(p, cknown);
     const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), total, tail, win, waste, known,
-                                 clip, cknown);
+                                 clip, cknown, cumulative_ratio(p),
+                                 ld_relaxed_u64(&p.ctl->g_first) >= p.startup_first ||
+                                     ld_relaxed_u32(&p.ctl->head_switches) >= 256u);
     const Head nhd{rehead(hd.h, k, d.k), pack_meta(hs, d.k, d.A, d.flo, d.since > 0xffff ? 0xffff : d.since)};
-    commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 2u);
+    commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 2u, d.flags);
 }
 
 // --------------------------------------------------------------- shared memory

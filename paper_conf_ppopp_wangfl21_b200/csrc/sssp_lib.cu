@@ -71,7 +71,9 @@ struct sssp_graph {
     uint2* d_adj = nullptr;
     uint64_t sum_w = 0;
     uint32_t max_w = 0;
-    uint32_t heur_k = 0;
+    uint32_t heur_k_span = 0;  // log2 initial Delta, max_w / B rule (ring span)
+    uint32_t heur_k_md = 0;    // log2 initial Delta, max_w / D rule
+    uint32_t heur_k_nf = 0;    // log2 initial Delta, Near-Far C*W/D rule
     sssp_options opts{};
     int sm_count = 0;
 
@@ -110,6 +112,7 @@ sssp_status check_options(const sssp_options& o) {
     if (o.num_buckets < 2 || o.num_buckets > 32 || (o.num_buckets & (o.num_buckets - 1)))
         return fail(SSSP_ERR_INVALID_ARGUMENT, "num_buckets must be a power of two in [2, 32]");
     if (o.delta_mode > 1) return fail(SSSP_ERR_INVALID_ARGUMENT, "delta_mode");
+    if (o.delta_heuristic > 2) return fail(SSSP_ERR_INVALID_ARGUMENT, "delta_heuristic");
     if (o.dist_bits != 0 && o.dist_bits != 32 && o.dist_bits != 64) return fail(SSSP_ERR_INVALID_ARGUMENT, "dist_bits");
     if (o.block_threads != 0 && o.block_threads != 128 && o.block_threads != 256 && o.block_threads != 512)
         return fail(SSSP_ERR_INVALID_ARGUMENT, "block_threads must be 0, 128, 256 or 512");
@@ -186,6 +189,7 @@ Params<DistT> make_params(sssp_graph* g, unsigned grid, unsigned bt, unsigned k_
     p.nb = g->opts.num_buckets;
     p.cap = g->cap;
     p.dynamic = g->opts.delta_mode == SSSP_DELTA_DYNAMIC;
+    p.adapt_active = (g->opts.flags & SSSP_FLAG_ADAPT_ACTIVE) ? 1u : 0u;
     p.clip_pct = g->opts.clip_pct;
     p.settle = g->opts.settle_head_switches;
     p.util_lo_pct = g->opts.util_lo_pct;
@@ -205,6 +209,7 @@ Params<DistT> make_params(sssp_graph* g, unsigned grid, unsigned bt, unsigned k_
     p.expanded = (unsigned*)g->expanded.p;
     p.waste_lo = g->opts.waste_lo_permille;
     p.waste_hi = g->opts.waste_hi_permille;
+    p.startup_first = (unsigned long long)g->n * g->opts.startup_permille / 1000ull;
     p.period_ns = (unsigned long long)(g->opts.period_us ? g->opts.period_us : 20u) * 1000ull;
     p.keep_frac = 0.0f;
     if (!(g->opts.flags & SSSP_FLAG_NO_L2_PERSIST) && g->persist_max) {
@@ -225,7 +230,7 @@ Params<DistT> make_params(sssp_graph* g, unsigned grid, unsigned bt, unsigned k_
 template <typename DistT>
 sssp_status launch_one(sssp_graph* g, uint32_t source, unsigned long long* out_dev, cudaStream_t s, int bits,
                        unsigned k0) {
-    const unsigned bt = g->opts.block_threads ? g->opts.block_threads : 256;
+    const unsigned bt = g->opts.block_threads ? g->opts.block_threads : 512;
     const KVariant kv = persistent_variant(bits, (int)bt);
     void* fn = kv.fn;
     CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kv.smem), "smem attribute");
@@ -259,8 +264,16 @@ sssp_status launch_one(sssp_graph* g, uint32_t source, unsigned long long* out_d
     return SSSP_OK;
 }
 
+unsigned heuristic_k(const sssp_graph* g) {
+    switch (g->opts.delta_heuristic) {
+        case SSSP_DELTA_H_NEARFAR: return g->heur_k_nf;
+        case SSSP_DELTA_H_MAXW_OVER_D: return g->heur_k_md;
+        default: return std::min(ilog2_round((double)g->max_w / (double)g->opts.num_buckets), 63u);
+    }
+}
+
 sssp_status launch_attempt(sssp_graph* g, uint32_t source, unsigned long long* out_dev, cudaStream_t s, int bits) {
-    const unsigned k0 = g->opts.delta_init ? ilog2_round((double)g->opts.delta_init) : g->heur_k;
+    const unsigned k0 = g->opts.delta_init ? ilog2_round((double)g->opts.delta_init) : heuristic_k(g);
     sssp_status st = ensure_ring(g, bits == 32 ? 8 : 16, g->cap ? g->cap : default_cap(g));
     if (st) return st;
     if ((st = ensure_trace(g))) return st;
@@ -413,9 +426,10 @@ void sssp_options_default(sssp_options* o) {
     o->settle_head_switches = 8;   // P:215 (reading R7): controller steps between Delta changes
     o->util_lo_pct = 100;          // P:211 (reading R6)
     o->util_hi_pct = 400;
-    o->waste_lo_permille = 50;     // reading R6: grow Delta only while < 5% of expansions are repeats
+    o->waste_lo_permille = 350;    // reading R6: grow Delta only while < 35% of expansions are repeats
     o->waste_hi_permille = 500;    //             shrink it while > 50% are (work <~ 2x Dijkstra)
     o->period_us = 20;
+    o->startup_permille = 2;
     o->dist_bits = 0;
     o->ring_items = 0;
     o->flags = 0;
@@ -510,11 +524,14 @@ sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offset
         return bail(fail(SSSP_ERR_INVALID_GRAPH, "col[" + std::to_string(scr[1]) + "] >= n"));
     g->sum_w = scr[2];
     g->max_w = (uint32_t)scr[3];
-    // initial Delta: C * W / D with W = average weight, D = average degree, C = 32 (reading R3)
+    // initial Delta (reading R3): max_w / D (Meyer-Sanders' Theta(1/d) rule for Delta-stepping [15]),
+    // or the Near-Far rule C * W / D with W = average weight, D = average degree, C = 32
     if (m && g->sum_w) {
         const double W = (double)g->sum_w / (double)m, D = (double)m / (double)n;
-        g->heur_k = std::min(ilog2_round(32.0 * W / D), 63u);
+        g->heur_k_nf = std::min(ilog2_round(32.0 * W / D), 63u);
+        g->heur_k_md = std::min(ilog2_round((double)g->max_w / std::max(D, 1.0)), 63u);
     }
+    g->heur_k_span = std::min(ilog2_round((double)g->max_w / (double)o.num_buckets), 63u);
     // 32-bit distances are provably safe when (n-1) * max_w < 2^32 - 1; otherwise
     // they are tried first and the overflow flag triggers a 64-bit re-run.
     g->cur_bits = 32;
@@ -640,7 +657,7 @@ sssp_status sssp_graph_info(const sssp_graph* g, uint32_t* n, uint64_t* m, uint6
     if (m) *m = g->m;
     if (sum_w) *sum_w = g->sum_w;
     if (max_w) *max_w = g->max_w;
-    if (heuristic_delta_log2) *heuristic_delta_log2 = g->heur_k;
+    if (heuristic_delta_log2) *heuristic_delta_log2 = heuristic_k(g);
     return SSSP_OK;
 }
 

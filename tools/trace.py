@@ -38,7 +38,7 @@ def main():
     for e in tr[::step]:
         print(f'{(e["time_ns"] - t0) / 1e3:9.1f}us head={e["head"]:8d} k={e["delta_log2"]:2d} A={e["active"]:2d} '
               f'pend={e["pending_total"]:9d} win={e["pending_window"]:9d} tail={e["pending_tail"]:8d} '
-              f'waste={e["waste_permille"]:4d} why={e["reason"]}')
+              f'waste={e["waste_permille"]:4d} why={e["reason"] & 255} flags={e["reason"] >> 8:09b}')
 
 
 if __name__ == "__main__":
