@@ -113,7 +113,7 @@ typedef struct sssp_options {
     uint64_t ring_items;       /* capacity of each bucket's circular array (items, rounded up to a
                                   power of two, >= 64); 0 = auto = max(2^16, next_pow2(n)) */
     uint32_t flags;            /* SSSP_FLAG_* */
-    uint32_t block_threads;    /* worker CTA size: 0 = auto (512), else 128/256/512 */
+    uint32_t block_threads;    /* worker CTA size: 0 = auto (512), else 128/256/512/1024 */
     uint32_t grid_ctas;        /* 0 = every co-resident CTA; else at most this many CTAs */
     uint32_t batch_min;        /* minimum items a CTA claims when enough are available; 0 = auto */
     uint32_t timeout_ms;       /* device watchdog (globaltimer); 0 = default 60000 */

@@ -22,7 +22,7 @@ import numpy as np
 
 from . import _build
 
-LIB_PATH = _build.LIB
+LIB_PATH = os.environ.get("SSSP_LIB", _build.LIB)  # override only for A/B experiments (tools/)
 _lib = None
 
 INF = 0xFFFFFFFFFFFFFFFF

@@ -384,13 +384,20 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
             // -------------------------------------------------------- claim
             if (warp == 0) {
                 int cmd = CMD_IDLE;
-                // one round trip: status, head, every bucket's avail gate
-                const unsigned st = ld_relaxed_u32(&p.ctl->status);
-                const Head hd = ld_head(&p.ctl->head);
-                const long long av_abs = lane < (int)p.nb ? (long long)ld_relaxed_u64(&p.bk[lane].avail.v) : 0;
+                // status + head (lane 0), then only the A active buckets' avail gates:
+                // idle CTAs poll here, so every extra line read lands on a hot L2 slice
+                unsigned st = 0;
+                Head hd{0ull, 0ull};
+                if (lane == 0) {
+                    st = ld_relaxed_u32(&p.ctl->status);
+                    hd = ld_head(&p.ctl->head);
+                }
+                st = __shfl_sync(FULL, st, 0);
+                hd.h = __shfl_sync(FULL, hd.h, 0);
+                hd.meta = __shfl_sync(FULL, hd.meta, 0);
                 const unsigned hs = meta_hs(hd.meta), A = meta_A(hd.meta);
-                long long av = __shfl_sync(FULL, av_abs, (hs + lane) & nbm);
-                if (lane >= (int)A) av = 0;
+                long long av = 0;
+                if (lane < (int)A && !st) av = (long long)ld_relaxed_u64(&p.bk[(hs + lane) & nbm].avail.v);
                 if (st) {
                     cmd = CMD_EXIT;
                 } else {

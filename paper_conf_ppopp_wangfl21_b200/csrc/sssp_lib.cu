@@ -114,8 +114,9 @@ sssp_status check_options(const sssp_options& o) {
     if (o.delta_mode > 1) return fail(SSSP_ERR_INVALID_ARGUMENT, "delta_mode");
     if (o.delta_heuristic > 2) return fail(SSSP_ERR_INVALID_ARGUMENT, "delta_heuristic");
     if (o.dist_bits != 0 && o.dist_bits != 32 && o.dist_bits != 64) return fail(SSSP_ERR_INVALID_ARGUMENT, "dist_bits");
-    if (o.block_threads != 0 && o.block_threads != 128 && o.block_threads != 256 && o.block_threads != 512)
-        return fail(SSSP_ERR_INVALID_ARGUMENT, "block_threads must be 0, 128, 256 or 512");
+    if (o.block_threads != 0 && o.block_threads != 128 && o.block_threads != 256 && o.block_threads != 512 &&
+        o.block_threads != 1024)
+        return fail(SSSP_ERR_INVALID_ARGUMENT, "block_threads must be 0, 128, 256, 512 or 1024");
     if (o.clip_pct == 0 || o.clip_pct > 100) return fail(SSSP_ERR_INVALID_ARGUMENT, "clip_pct");
     if (o.active_init > o.num_buckets) return fail(SSSP_ERR_INVALID_ARGUMENT, "active_init > num_buckets");
     if (o.waste_lo_permille > 1000 || o.waste_hi_permille > 1000) return fail(SSSP_ERR_INVALID_ARGUMENT, "waste permille");
@@ -132,17 +133,19 @@ struct KVariant {
 };
 template <typename DistT, int BT>
 KVariant kvar() {
-    constexpr int W = BT >= 256 ? 2048 : 1024;
+    constexpr int W = BT >= 1024 ? 4096 : (BT >= 256 ? 2048 : 1024);
     return KVariant{(void*)adds_persistent_kernel<DistT, BT, 4, W>, Smem<DistT, BT, 4, W>::bytes};
 }
 KVariant persistent_variant(int bits, int bt) {
     if (bits == 32) {
         if (bt == 128) return kvar<uint32_t, 128>();
         if (bt == 512) return kvar<uint32_t, 512>();
+        if (bt == 1024) return kvar<uint32_t, 1024>();
         return kvar<uint32_t, 256>();
     }
     if (bt == 128) return kvar<unsigned long long, 128>();
     if (bt == 512) return kvar<unsigned long long, 512>();
+    if (bt == 1024) return kvar<unsigned long long, 1024>();
     return kvar<unsigned long long, 256>();
 }
 
