@@ -120,7 +120,8 @@ typedef struct sssp_options {
     uint32_t trace_capacity;   /* trace ring entries when SSSP_FLAG_TRACE; 0 = 65536 */
     uint32_t active_init;      /* initial number of active (claimable) buckets; 0 = auto (1) */
     uint32_t local_max;        /* head-bucket children a CTA keeps as its own next batch instead of
-                                  publishing them (0 = auto = block_threads; see SSSP_FLAG_NO_LOCAL) */
+                                  publishing them, when its batch was at most half a CTA (latency regime);
+                                  0 = auto = 128; see SSSP_FLAG_NO_LOCAL */
     uint32_t max_backoff_ns;   /* idle CTAs back off exponentially up to this (0 = auto = 2048) */
     uint32_t startup_permille; /* the controller may not grow Delta before this share of the vertices
                                   has been expanded or 256 head switches have happened (start-up

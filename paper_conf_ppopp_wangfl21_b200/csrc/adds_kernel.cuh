@@ -458,6 +458,11 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
             from_ring = true;
         }
 
+        // CTA-local continuation only in the latency regime (small batches = scarce
+        // work): with plentiful work it starves the other CTAs of head-bucket items
+        // (measured: RMAT 2x slower with a full-CTA cap)
+        const unsigned lcap = got * 2 <= (unsigned)BT ? local_max : 0u;
+
         // ------------------------------------------------------------ pop + stale check
         const Head hd = s_head;
         const unsigned hs = meta_hs(hd.meta), k = meta_k(hd.meta);
@@ -645,14 +650,14 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                     const unsigned o = push[j] ? adds_bucket_offset(nd[j], k, hd.h, p.nb) : 0u;
                     // head-bucket children stay in this CTA (warp-aggregated slot grab)
                     bool kept = false;
-                    if (local_max) {
+                    if (lcap) {
                         const unsigned lm = __ballot_sync(FULL, push[j] && o == 0);
                         if (lm) {
                             const int leader = __ffs(lm) - 1;
                             unsigned pos = 0;
                             if (lane == leader) pos = atomicAdd(&s_lnext, (unsigned)__popc(lm));
                             pos = __shfl_sync(FULL, pos, leader) + __popc(lm & lt_mask);
-                            if (push[j] && o == 0 && pos < local_max) {
+                            if (push[j] && o == 0 && pos < lcap) {
                                 s_lv[pos] = a[j].x;
                                 s_ld[pos] = (DistT)nd[j];
                                 kept = true;
@@ -749,7 +754,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
 
         // ------------------------------------------------------------ complete
         __syncthreads();  // s_lnext final (also covers the E == 0 case)
-        const unsigned kept = s_lnext < local_max ? s_lnext : local_max;
+        const unsigned kept = s_lnext < lcap ? s_lnext : lcap;
         if (tid == 0) {
             // one atomic: the kept children inherit the parents' accounting
             if (got > kept) atomicAdd(&p.bk[slot].done.v, (unsigned long long)(got - kept));

@@ -204,7 +204,7 @@ Params<DistT> make_params(sssp_graph* g, unsigned grid, unsigned bt, unsigned k_
     unsigned sh = 0;
     while ((1u << (sh + 1)) <= grid) ++sh;  // floor(log2 grid)
     p.share_shift = sh > 2 ? sh - 2 : 0;
-    p.local_max = (g->opts.flags & SSSP_FLAG_NO_LOCAL) ? 0u : (g->opts.local_max ? g->opts.local_max : bt);
+    p.local_max = (g->opts.flags & SSSP_FLAG_NO_LOCAL) ? 0u : (g->opts.local_max ? g->opts.local_max : 128u);
     p.max_backoff_ns = g->opts.max_backoff_ns ? g->opts.max_backoff_ns : 2048u;
     p.prof = (g->opts.flags & SSSP_FLAG_PROFILE) ? 1u : 0u;
     // L2 residency of dist (D5): reserve the persisting set-aside for
