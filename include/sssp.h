@@ -98,7 +98,7 @@ typedef struct sssp_options {
     uint32_t util_lo_pct;      /* lower utilisation limit, % of resident threads; default 100 */
     uint32_t util_hi_pct;      /* upper utilisation limit, % of resident threads; default 400 */
     uint32_t waste_lo_permille;/* Delta may grow only while the recent re-expansion share is below this
-                                  (default 350 = 35%) */
+                                  (default 450 = 45%) */
     uint32_t waste_hi_permille;/* Delta shrinks (not below its clip floor) while the share is above this
                                   (default 500 = 50%, i.e. ~2x Dijkstra's vertex work) */
     uint32_t period_us;        /* periodic controller step (default 20 us; head switches also step) */
@@ -124,7 +124,7 @@ typedef struct sssp_options {
                                   0 = auto = 128; see SSSP_FLAG_NO_LOCAL */
     uint32_t max_backoff_ns;   /* idle CTAs back off exponentially up to this (0 = auto = 2048) */
     uint32_t startup_permille; /* the controller may not grow Delta before this share of the vertices
-                                  has been expanded or 256 head switches have happened (start-up
+                                  has been expanded or 32 head switches have happened (start-up
                                   frontiers are always small); default 2 */
     uint32_t reserved[1];
 } sssp_options;

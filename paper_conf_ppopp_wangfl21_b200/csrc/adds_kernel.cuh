@@ -97,7 +97,8 @@ __device__ __forceinline__ long long warp_sum_s64(long long x) {
 //   grow   window under-utilised AND share < lo   -> Delta x2
 //   A      active buckets follow the same two signals one step at a time
 // Settling: `since` counts controller steps (head switches and periodic
-// steps) since the last Delta change; a change needs since >= settle.
+// steps) since the last Delta change; a change needs since >= settle (a quarter
+// of that for growth while the re-expansion share is below waste_lo / 8).
 struct CtlDecision {
     unsigned k, A, flo, since;
     bool changed;
@@ -140,6 +141,9 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
             d.k = k + 1;
             d.changed = true;
         }
+    } else if (d.since * 4 >= p.settle && low && frugal && beyond && waste * 8 < p.waste_lo && k < p.k_max) {
+        d.k = k + 1;  // essentially no re-expansion yet: grow with a quarter of the settling time
+        d.changed = true;
     }
     if (d.changed) d.since = 0;
     // fine-grained knob: one more active bucket only when the hardware is
@@ -266,7 +270,7 @@ __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lan
     const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), total, tail, win, waste, known,
                                  clip, cknown, cumulative_ratio(p),
                                  ld_relaxed_u64(&p.ctl->g_first) >= p.startup_first ||
-                                     ld_relaxed_u32(&p.ctl->head_switches) >= 256u);
+                                     ld_relaxed_u32(&p.ctl->head_switches) >= 32u);
     const Head nhd{rehead(hd.h + o, k, d.k),
                    pack_meta((hs + o) & (nb - 1), d.k, d.A, d.flo, d.since > 0xffff ? 0xffff : d.since)};
     commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 1u, d.flags);
@@ -291,7 +295,7 @@ __device__ void periodic_step(const Params<DistT>& p, const int lane) {
     const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), total, tail, win, waste, known,
                                  clip, cknown, cumulative_ratio(p),
                                  ld_relaxed_u64(&p.ctl->g_first) >= p.startup_first ||
-                                     ld_relaxed_u32(&p.ctl->head_switches) >= 256u);
+                                     ld_relaxed_u32(&p.ctl->head_switches) >= 32u);
     const Head nhd{rehead(hd.h, k, d.k), pack_meta(hs, d.k, d.A, d.flo, d.since > 0xffff ? 0xffff : d.since)};
     commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 2u, d.flags);
 }

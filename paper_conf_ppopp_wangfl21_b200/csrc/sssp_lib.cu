@@ -429,7 +429,7 @@ void sssp_options_default(sssp_options* o) {
     o->settle_head_switches = 8;   // P:215 (reading R7): controller steps between Delta changes
     o->util_lo_pct = 100;          // P:211 (reading R6)
     o->util_hi_pct = 400;
-    o->waste_lo_permille = 350;    // reading R6: grow Delta only while < 35% of expansions are repeats
+    o->waste_lo_permille = 450;    // reading R6: grow Delta only while < 45% of expansions are repeats
     o->waste_hi_permille = 500;    //             shrink it while > 50% are (work <~ 2x Dijkstra)
     o->period_us = 20;
     o->startup_permille = 2;
