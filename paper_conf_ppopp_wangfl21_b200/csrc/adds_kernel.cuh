@@ -549,9 +549,15 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
             tw = 0;
         }
 
+        // latency fast path (road-like graphs): a batch whose arcs fit one round
+        // skips the owner map + async window and the L2 filter load -- two
+        // dependent steps fewer per hop; arcs are loaded directly, relaxed by atomicMin
+        const bool small = E <= (unsigned)kRound;
+        if (small) __syncthreads();  // publishes s_scan
         for (unsigned wbase = 0; wbase < E; wbase += W) {
             const unsigned Ew = (E - wbase) < (unsigned)W ? (E - wbase) : (unsigned)W;
             const long long tw0 = prof ? clock64() : 0;
+            if (!small) {
             // ------------------------------------------------ owner of every window position
             // zero, mark row starts, inclusive prefix-max (rows are in scan order)
             {
@@ -614,6 +620,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                 tw += clock64() - tw0;
                 s_prof[PR_N_WINDOW] += 1;
             }
+            }  // !small
 
             // ------------------------------------------------ relax + push (rounds)
             for (unsigned rbase = 0; rbase < Ew; rbase += kRound) {
@@ -621,20 +628,55 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                 unsigned long long nd[EPT];
                 bool push[EPT];
                 DistT cur[EPT];
+                if (small) {
+                    unsigned own[EPT];
 #pragma unroll
-                for (int j = 0; j < EPT; ++j) {
-                    const unsigned q = rbase + j * BT + tid;
-                    if (q < Ew) {
-                        a[j] = s_arc[q];
-                        nd[j] = (unsigned long long)s_d[s_owner[q]] + a[j].y;
-                    } else {
-                        a[j] = make_uint2(0u, 0u);
-                        nd[j] = kInf;
+                    for (int j = 0; j < EPT; ++j) {  // owner = largest i with scan[i] <= q
+                        const unsigned q = j * BT + tid;
+                        unsigned lo = 0, hi = got - 1;
+                        if (q < Ew) {
+                            while (lo < hi) {
+                                const unsigned mid = (lo + hi + 1) >> 1;
+                                if (s_scan[mid] <= q) lo = mid;
+                                else hi = mid - 1;
+                            }
+                        }
+                        own[j] = lo;
                     }
-                }
 #pragma unroll
-                for (int j = 0; j < EPT; ++j)  // EPT independent L2 gathers in flight
-                    cur[j] = nd[j] < kInf ? ld_keep(p.dist + a[j].x, pol_keep) : (DistT)0;
+                    for (int j = 0; j < EPT; ++j) {  // EPT independent arc loads in flight
+                        const unsigned q = j * BT + tid;
+                        if (q < Ew) {
+                            a[j] = ld_stream_u2(p.adj + s_ebeg[own[j]] + (q - s_scan[own[j]]), pol_stream);
+                            nd[j] = (unsigned long long)s_d[own[j]] + a[j].y;
+                            cur[j] = DistInf<DistT>::value;  // tiny batch: straight to atomicMin
+                        } else {
+                            a[j] = make_uint2(0u, 0u);
+                            nd[j] = kInf;
+                            cur[j] = (DistT)0;
+                        }
+                    }
+                    if (E > (unsigned)BT) {  // more than one arc per thread: keep the L2 filter
+#pragma unroll
+                        for (int j = 0; j < EPT; ++j)
+                            if (nd[j] < kInf) cur[j] = ld_keep(p.dist + a[j].x, pol_keep);
+                    }
+                } else {
+#pragma unroll
+                    for (int j = 0; j < EPT; ++j) {
+                        const unsigned q = rbase + j * BT + tid;
+                        if (q < Ew) {
+                            a[j] = s_arc[q];
+                            nd[j] = (unsigned long long)s_d[s_owner[q]] + a[j].y;
+                        } else {
+                            a[j] = make_uint2(0u, 0u);
+                            nd[j] = kInf;
+                        }
+                    }
+#pragma unroll
+                    for (int j = 0; j < EPT; ++j)  // EPT independent L2 gathers in flight
+                        cur[j] = nd[j] < kInf ? ld_keep(p.dist + a[j].x, pol_keep) : (DistT)0;
+                }
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {
                     const unsigned q = rbase + j * BT + tid;
