@@ -242,3 +242,13 @@ def test_run_batch_distributed_single_rank():
     for i, s in enumerate(srcs):
         assert np.array_equal(full[i], oracle.dijkstra(g, int(s))[0])
     assert out["stats"]["runs"] == 5
+
+
+def test_loaded_file_through_the_abi(tmp_path):
+    from graphgen import loaders
+    g = gg.make("road", scale_down=10)
+    p = str(tmp_path / "road.gr")
+    loaders.save_galois_gr(g, p)
+    h = loaders.load(p)
+    s = int(gg.config_sources("road", h, 1)[0])
+    check(h, s)
