@@ -76,6 +76,10 @@ typedef enum sssp_status {
                                         By default a run raises cudaLimitPersistingL2CacheSize (device-wide)
                                         up to min(dist bytes, device maximum) */
 
+/* Algorithms (options.algorithm) */
+#define SSSP_ALGO_ADDS 0u
+#define SSSP_ALGO_NEAR_FAR 1u
+
 /* Initial-Delta heuristics (options.delta_heuristic) */
 #define SSSP_DELTA_H_RING_SPAN 0u
 #define SSSP_DELTA_H_MAXW_OVER_D 2u
@@ -126,7 +130,13 @@ typedef struct sssp_options {
     uint32_t startup_permille; /* the controller may not grow Delta before this share of the vertices
                                   has been expanded or 32 head switches have happened (start-up
                                   frontiers are always small); default 2 */
-    uint32_t reserved[1];
+    uint32_t concurrent_sources; /* sssp_run_batch: sources in flight at once on this GPU (NEXT-1), each
+                                  with its own workspace (dist, bucket ring, counters) and stream and
+                                  1/c of the SMs; the CSR is shared.  0/1 = one at a time */
+    uint32_t algorithm;        /* SSSP_ALGO_ADDS (default) or SSSP_ALGO_NEAR_FAR: the paper's comparison
+                                  system as an ablation -- 2 buckets, static Delta (default the
+                                  Near-Far rule C*W/D), bulk-synchronous double-buffered piles */
+    uint32_t reserved2[3];
 } sssp_options;
 
 typedef struct sssp_stats {
@@ -150,7 +160,9 @@ typedef struct sssp_stats {
     float kernel_ms;             /* device time of the persistent kernel(s) (CUDA events) */
     float total_ms;              /* device time init + kernel + finalize (CUDA events) */
     uint32_t status;             /* sssp_status of the last run (for SSSP_FLAG_ASYNC) */
-    uint32_t reserved[3];
+    float batch_ms;              /* device time of the whole call on the caller's stream (CUDA events) */
+    uint32_t concurrency;        /* sources that were in flight at once */
+    uint32_t reserved[1];
 } sssp_stats;
 
 /* One Delta-controller sample (written at each head-bucket switch and at each
@@ -206,8 +218,10 @@ sssp_status sssp_run(sssp_graph *g, uint32_t source, uint64_t *dist_out, sssp_st
 
 /* Multi-source batch: k sources (host array), results row-major
  * dist_out[i*n + v] for source i (k*n uint64 entries, device or host).
- * Equivalent to k calls of sssp_run (bit-identical), amortising launch and
- * status overheads; stats cover the whole batch.  Errors as sssp_run plus
+ * Equivalent to k calls of sssp_run (bit-identical); with
+ * options.concurrent_sources = c > 1 up to c sources run concurrently (each
+ * with its own workspace and stream, joined back to `stream` before return).
+ * Stats cover the whole batch (batch_ms = device time of the call).  Errors as sssp_run plus
  * INVALID_ARGUMENT for k == 0 or any source >= n (checked before any work). */
 sssp_status sssp_run_batch(sssp_graph *g, const uint32_t *sources, uint32_t k,
                            uint64_t *dist_out, sssp_stream_t stream);

@@ -37,6 +37,8 @@ SSSP_FLAG_ADAPT_ACTIVE = 0x40
 PROFILE_FIELDS = ["cyc_claim", "cyc_idle", "cyc_pop", "cyc_scan", "cyc_rounds", "cyc_flush", "cyc_complete",
                   "cyc_total", "n_ring_batches", "n_local_batches", "n_idle", "n_flush", "n_rounds", "n_ctas",
                   "cyc_window", "n_windows"]
+SSSP_ALGO_ADDS = 0
+SSSP_ALGO_NEAR_FAR = 1
 SSSP_DELTA_H_RING_SPAN = 0
 SSSP_DELTA_H_NEARFAR = 1
 SSSP_DELTA_H_MAXW_OVER_D = 2
@@ -69,7 +71,8 @@ class sssp_options(ctypes.Structure):
         ("flags", ctypes.c_uint32), ("block_threads", ctypes.c_uint32), ("grid_ctas", ctypes.c_uint32),
         ("batch_min", ctypes.c_uint32), ("timeout_ms", ctypes.c_uint32), ("trace_capacity", ctypes.c_uint32),
         ("active_init", ctypes.c_uint32), ("local_max", ctypes.c_uint32), ("max_backoff_ns", ctypes.c_uint32),
-        ("startup_permille", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 1),
+        ("startup_permille", ctypes.c_uint32), ("concurrent_sources", ctypes.c_uint32),
+        ("algorithm", ctypes.c_uint32), ("reserved2", ctypes.c_uint32 * 3),
     ]
 
 
@@ -81,7 +84,8 @@ class sssp_stats(ctypes.Structure):
         ("head_switches", ctypes.c_uint32), ("delta_changes", ctypes.c_uint32), ("retries", ctypes.c_uint32),
         ("dist_bits", ctypes.c_uint32), ("grid_ctas", ctypes.c_uint32), ("block_threads", ctypes.c_uint32),
         ("runs", ctypes.c_uint32), ("trace_entries", ctypes.c_uint32), ("kernel_ms", ctypes.c_float),
-        ("total_ms", ctypes.c_float), ("status", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3),
+        ("total_ms", ctypes.c_float), ("status", ctypes.c_uint32), ("batch_ms", ctypes.c_float),
+        ("concurrency", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 1),
     ]
 
 

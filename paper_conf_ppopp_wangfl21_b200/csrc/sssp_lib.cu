@@ -8,10 +8,12 @@
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <vector>
 
 #include "../../include/sssp.h"
 #include "adds_kernel.cuh"
 #include "aux_kernels.cuh"
+#include "nearfar_kernel.cuh"
 #include "bucket_map.h"
 
 using namespace adds;
@@ -63,6 +65,40 @@ struct DevBuf {
 
 }  // namespace
 
+// One run's device state: a graph handle owns one workspace per concurrently
+// running source (NEXT-1); workspace 0 runs on the caller's stream.
+struct Workspace {
+    DevBuf dist;        // 8n bytes (serves 32- and 64-bit distances)
+    DevBuf ring;        // nb * cap * item bytes
+    DevBuf bk, ctl, trace, expanded;
+    unsigned long long cap = 0;
+    int ring_item_bytes = 0;
+    unsigned trace_alloc = 0;
+    Ctl* h_ctl = nullptr;  // pinned status block
+    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+    cudaStream_t own_stream = nullptr;  // slots > 0
+    DevBuf nf_piles, nf_cnt;            // Near-Far ablation: 4 pile buffers + counters
+    unsigned long long nf_cap = 0;
+    int nf_item_bytes = 0;
+    uint32_t last_grid = 0, last_block = 0, last_k0 = 0;
+    void release() {
+        dist.release();
+        ring.release();
+        bk.release();
+        ctl.release();
+        trace.release();
+        expanded.release();
+        nf_piles.release();
+        nf_cnt.release();
+        if (h_ctl) cudaFreeHost(h_ctl);
+        h_ctl = nullptr;
+        for (auto& e : ev)
+            if (e) cudaEventDestroy(e);
+        if (own_stream) cudaStreamDestroy(own_stream);
+        own_stream = nullptr;
+    }
+};
+
 struct sssp_graph {
     int device = 0;
     uint32_t n = 0;
@@ -76,22 +112,14 @@ struct sssp_graph {
     uint32_t heur_k_nf = 0;    // log2 initial Delta, Near-Far C*W/D rule
     sssp_options opts{};
     int sm_count = 0;
-
-    DevBuf dist;        // 8n bytes (serves 32- and 64-bit distances)
-    DevBuf ring;        // nb * cap * item bytes
-    unsigned long long cap = 0;
-    int ring_item_bytes = 0;
-    DevBuf bk, ctl, trace, scratch, hostout, expanded;
-    unsigned trace_alloc = 0;
-    Ctl* h_ctl = nullptr;  // pinned
-    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
-
-    int cur_bits = 32;  // 64 after a 32-bit overflow was observed (sticky)
+    std::vector<Workspace*> ws;
+    DevBuf scratch, hostout;
+    cudaEvent_t bev[2] = {nullptr, nullptr};  // batch start / end on the caller's stream
+    int cur_bits = 32;       // 64 after a 32-bit overflow was observed (sticky)
     size_t persist_max = 0;  // device's L2 persisting set-aside limit (bytes)
     bool busy = false;
     bool async_pending = false;
     sssp_stats stats{};
-    uint32_t last_grid = 0, last_block = 0, last_k0 = 0;
 };
 
 namespace {
@@ -120,6 +148,8 @@ sssp_status check_options(const sssp_options& o) {
     if (o.clip_pct == 0 || o.clip_pct > 100) return fail(SSSP_ERR_INVALID_ARGUMENT, "clip_pct");
     if (o.active_init > o.num_buckets) return fail(SSSP_ERR_INVALID_ARGUMENT, "active_init > num_buckets");
     if (o.waste_lo_permille > 1000 || o.waste_hi_permille > 1000) return fail(SSSP_ERR_INVALID_ARGUMENT, "waste permille");
+    if (o.concurrent_sources > 64) return fail(SSSP_ERR_INVALID_ARGUMENT, "concurrent_sources > 64");
+    if (o.algorithm > SSSP_ALGO_NEAR_FAR) return fail(SSSP_ERR_INVALID_ARGUMENT, "algorithm");
     return SSSP_OK;
 }
 
@@ -149,48 +179,79 @@ KVariant persistent_variant(int bits, int bt) {
     return kvar<unsigned long long, 256>();
 }
 
-sssp_status ensure_ring(sssp_graph* g, int item_bytes, unsigned long long cap) {
-    const size_t bytes = (size_t)g->opts.num_buckets * cap * item_bytes;
-    if (g->ring.p && g->ring.bytes >= bytes && g->cap == cap && g->ring_item_bytes == item_bytes) return SSSP_OK;
-    g->ring.release();
-    CK(cudaMalloc(&g->ring.p, bytes), "allocating the bucket ring");
-    g->ring.bytes = bytes;
-    CK(cudaMemset(g->ring.p, 0xFF, bytes), "clearing the bucket ring");
-    g->cap = cap;
-    g->ring_item_bytes = item_bytes;
-    return SSSP_OK;
-}
-
-sssp_status ensure_trace(sssp_graph* g) {
-    if (!(g->opts.flags & SSSP_FLAG_TRACE)) return SSSP_OK;
-    unsigned cap = g->opts.trace_capacity ? g->opts.trace_capacity : 65536u;
-    if (g->trace.p && g->trace_alloc >= cap) return SSSP_OK;
-    g->trace.release();
-    CK(cudaMalloc(&g->trace.p, (size_t)cap * sizeof(TraceEntry)), "allocating the trace ring");
-    g->trace_alloc = cap;
-    return SSSP_OK;
-}
-
 unsigned long long default_cap(const sssp_graph* g) {
     if (g->opts.ring_items) return next_pow2(std::max<unsigned long long>(g->opts.ring_items, 64ull));
     return next_pow2(std::max<unsigned long long>((unsigned long long)g->n, 1ull << 16));
 }
 
+sssp_status ensure_ring(sssp_graph* g, Workspace& w, int item_bytes, unsigned long long cap) {
+    const size_t bytes = (size_t)g->opts.num_buckets * cap * item_bytes;
+    if (w.ring.p && w.ring.bytes >= bytes && w.cap == cap && w.ring_item_bytes == item_bytes) return SSSP_OK;
+    w.ring.release();
+    CK(cudaMalloc(&w.ring.p, bytes), "allocating the bucket ring");
+    w.ring.bytes = bytes;
+    CK(cudaMemset(w.ring.p, 0xFF, bytes), "clearing the bucket ring");
+    w.cap = cap;
+    w.ring_item_bytes = item_bytes;
+    return SSSP_OK;
+}
+
+sssp_status ensure_trace(sssp_graph* g, Workspace& w) {
+    if (!(g->opts.flags & SSSP_FLAG_TRACE)) return SSSP_OK;
+    unsigned cap = g->opts.trace_capacity ? g->opts.trace_capacity : 65536u;
+    if (w.trace.p && w.trace_alloc >= cap) return SSSP_OK;
+    w.trace.release();
+    CK(cudaMalloc(&w.trace.p, (size_t)cap * sizeof(TraceEntry)), "allocating the trace ring");
+    w.trace_alloc = cap;
+    return SSSP_OK;
+}
+
+sssp_status alloc_workspace(sssp_graph* g, Workspace& w, bool own_stream) {
+    const size_t n = g->n;
+    CK(cudaMalloc(&w.dist.p, n * 8), "allocating dist");
+    w.dist.bytes = n * 8;
+    CK(cudaMalloc(&w.expanded.p, (n + 31) / 32 * 4), "allocating the expansion bitmap");
+    CK(cudaMalloc(&w.bk.p, sizeof(BucketCtl) * kMaxBuckets), "allocating bucket counters");
+    CK(cudaMemset(w.bk.p, 0, sizeof(BucketCtl) * kMaxBuckets), "bucket counters");
+    CK(cudaMalloc(&w.ctl.p, sizeof(Ctl)), "allocating control block");
+    CK(cudaMemset(w.ctl.p, 0, sizeof(Ctl)), "control block");
+    CK(cudaHostAlloc((void**)&w.h_ctl, sizeof(Ctl), cudaHostAllocDefault), "allocating pinned status block");
+    std::memset(w.h_ctl, 0, sizeof(Ctl));
+    for (auto& e : w.ev) CK(cudaEventCreate(&e), "creating events");
+    if (own_stream) CK(cudaStreamCreateWithFlags(&w.own_stream, cudaStreamNonBlocking), "creating a slot stream");
+    return ensure_ring(g, w, (g->opts.dist_bits == 64) ? 16 : 8, default_cap(g));
+}
+
+sssp_status ensure_slots(sssp_graph* g, unsigned c) {
+    while (g->ws.size() < c) {
+        Workspace* w = new Workspace();
+        g->ws.push_back(w);
+        sssp_status st = alloc_workspace(g, *w, g->ws.size() > 1);
+        if (st) {
+            w->release();
+            delete w;
+            g->ws.pop_back();
+            return st;
+        }
+    }
+    return SSSP_OK;
+}
+
 template <typename DistT>
-Params<DistT> make_params(sssp_graph* g, unsigned grid, unsigned bt, unsigned k_max) {
+Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned bt, unsigned k_max, unsigned conc) {
     Params<DistT> p{};
     p.off = g->d_off;
     p.adj = g->d_adj;
-    p.dist = (DistT*)g->dist.p;
-    p.ring = (char*)g->ring.p;
-    p.bk = (BucketCtl*)g->bk.p;
-    p.ctl = (Ctl*)g->ctl.p;
+    p.dist = (DistT*)w.dist.p;
+    p.ring = (char*)w.ring.p;
+    p.bk = (BucketCtl*)w.bk.p;
+    p.ctl = (Ctl*)w.ctl.p;
     const bool tr = (g->opts.flags & SSSP_FLAG_TRACE) != 0;
-    p.trace = tr ? (TraceEntry*)g->trace.p : nullptr;
-    p.trace_cap = tr ? g->trace_alloc : 0;
+    p.trace = tr ? (TraceEntry*)w.trace.p : nullptr;
+    p.trace_cap = tr ? w.trace_alloc : 0;
     p.n = g->n;
     p.nb = g->opts.num_buckets;
-    p.cap = g->cap;
+    p.cap = w.cap;
     p.dynamic = g->opts.delta_mode == SSSP_DELTA_DYNAMIC;
     p.adapt_active = (g->opts.flags & SSSP_FLAG_ADAPT_ACTIVE) ? 1u : 0u;
     p.clip_pct = g->opts.clip_pct;
@@ -207,16 +268,17 @@ Params<DistT> make_params(sssp_graph* g, unsigned grid, unsigned bt, unsigned k_
     p.local_max = (g->opts.flags & SSSP_FLAG_NO_LOCAL) ? 0u : (g->opts.local_max ? g->opts.local_max : 128u);
     p.max_backoff_ns = g->opts.max_backoff_ns ? g->opts.max_backoff_ns : 2048u;
     p.prof = (g->opts.flags & SSSP_FLAG_PROFILE) ? 1u : 0u;
-    // L2 residency of dist (DESIGN.md D5): reserve the persisting set-aside for
-    // it and mark dist accesses evict_last over the fraction that fits
-    p.expanded = (unsigned*)g->expanded.p;
+    p.expanded = (unsigned*)w.expanded.p;
     p.waste_lo = g->opts.waste_lo_permille;
     p.waste_hi = g->opts.waste_hi_permille;
     p.startup_first = (unsigned long long)g->n * g->opts.startup_permille / 1000ull;
     p.period_ns = (unsigned long long)(g->opts.period_us ? g->opts.period_us : 20u) * 1000ull;
+    // L2 residency of dist (DESIGN.md D5): reserve the persisting set-aside for
+    // the concurrently live dist arrays and mark dist accesses evict_last over
+    // the fraction that fits
     p.keep_frac = 0.0f;
     if (!(g->opts.flags & SSSP_FLAG_NO_L2_PERSIST) && g->persist_max) {
-        const size_t want = (size_t)g->n * sizeof(DistT);
+        const size_t want = (size_t)g->n * sizeof(DistT) * conc;
         const size_t use = std::min(want, g->persist_max);
         size_t cur = 0;
         cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
@@ -229,10 +291,21 @@ Params<DistT> make_params(sssp_graph* g, unsigned grid, unsigned bt, unsigned k_
     return p;
 }
 
-// One attempt of one source with `bits`-wide internal distances.
+unsigned heuristic_k(const sssp_graph* g) {
+    switch (g->opts.delta_heuristic) {
+        case SSSP_DELTA_H_NEARFAR: return g->heur_k_nf;
+        case SSSP_DELTA_H_MAXW_OVER_D: return g->heur_k_md;
+        default: return std::min(ilog2_round((double)g->max_w / (double)g->opts.num_buckets), 63u);
+    }
+}
+
+// One attempt of one source with `bits`-wide internal distances on workspace w.
+// `conc` workspaces share the GPU: each persistent grid gets 1/conc of the CTAs.
+// (The kernel never waits on a CTA that has not started -- no grid barrier --
+// so co-residency is not required; one slot launches cooperatively anyway.)
 template <typename DistT>
-sssp_status launch_one(sssp_graph* g, uint32_t source, unsigned long long* out_dev, cudaStream_t s, int bits,
-                       unsigned k0) {
+sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, unsigned long long* out_dev, cudaStream_t s,
+                       int bits, unsigned k0, unsigned conc) {
     const unsigned bt = g->opts.block_threads ? g->opts.block_threads : 512;
     const KVariant kv = persistent_variant(bits, (int)bt);
     void* fn = kv.fn;
@@ -242,49 +315,109 @@ sssp_status launch_one(sssp_graph* g, uint32_t source, unsigned long long* out_d
     if (occ < 1) return fail(SSSP_ERR_CUDA, "persistent kernel cannot be resident");
     unsigned grid = (unsigned)(occ * g->sm_count);
     if (g->opts.grid_ctas && g->opts.grid_ctas < grid) grid = g->opts.grid_ctas;
+    grid = std::max(1u, grid / conc);
     const unsigned k_max = bits == 32 ? 31u : 63u;
     unsigned k = std::min(k0, k_max);
     const unsigned A0 = g->opts.active_init ? g->opts.active_init : 1u;
     Head h0{0ull, pack_meta(0, k, A0, 0, 0)};
-    Params<DistT> p = make_params<DistT>(g, grid, bt, k_max);
+    Params<DistT> p = make_params<DistT>(g, w, grid, bt, k_max, conc);
 
-    const unsigned aux_grid = (unsigned)g->sm_count * 8;
-    CK(cudaEventRecord(g->ev[0], s), "event");
-    init_run_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, g->n, source, p.ctl, p.bk, p.ring, g->cap, h0,
+    const unsigned aux_grid = (unsigned)g->sm_count * 8 / conc + 1;
+    CK(cudaEventRecord(w.ev[0], s), "event");
+    init_run_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, g->n, source, p.ctl, p.bk, p.ring, w.cap, h0,
                                                     p.expanded);
     CK(cudaGetLastError(), "init kernel launch");
-    CK(cudaEventRecord(g->ev[1], s), "event");
+    CK(cudaEventRecord(w.ev[1], s), "event");
     void* args[] = {(void*)&p};
-    CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(bt), args, kv.smem, s), "persistent kernel launch");
-    CK(cudaEventRecord(g->ev[2], s), "event");
+    if (conc == 1) {
+        CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(bt), args, kv.smem, s), "persistent kernel launch");
+    } else {
+        CK(cudaLaunchKernel(fn, dim3(grid), dim3(bt), args, kv.smem, s), "persistent kernel launch");
+    }
+    CK(cudaEventRecord(w.ev[2], s), "event");
     finalize_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, out_dev, g->n, g->d_off, p.ctl);
     CK(cudaGetLastError(), "finalize kernel launch");
-    CK(cudaEventRecord(g->ev[3], s), "event");
-    CK(cudaMemcpyAsync(g->h_ctl, g->ctl.p, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "status copy");
-    g->last_grid = grid;
-    g->last_block = bt;
-    g->last_k0 = k;
+    CK(cudaEventRecord(w.ev[3], s), "event");
+    CK(cudaMemcpyAsync(w.h_ctl, w.ctl.p, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "status copy");
+    w.last_grid = grid;
+    w.last_block = bt;
+    w.last_k0 = k;
     return SSSP_OK;
 }
 
-unsigned heuristic_k(const sssp_graph* g) {
-    switch (g->opts.delta_heuristic) {
-        case SSSP_DELTA_H_NEARFAR: return g->heur_k_nf;
-        case SSSP_DELTA_H_MAXW_OVER_D: return g->heur_k_md;
-        default: return std::min(ilog2_round((double)g->max_w / (double)g->opts.num_buckets), 63u);
-    }
+// ------------------------------------------------------------ Near-Far ablation (NEXT-2)
+sssp_status ensure_nf(sssp_graph* g, Workspace& w, int item_bytes, unsigned long long cap) {
+    if (w.nf_piles.p && w.nf_cap == cap && w.nf_item_bytes == item_bytes) return SSSP_OK;
+    w.nf_piles.release();
+    CK(cudaMalloc(&w.nf_piles.p, 4 * (size_t)cap * item_bytes), "allocating Near-Far piles");
+    w.nf_piles.bytes = 4 * (size_t)cap * item_bytes;
+    if (!w.nf_cnt.p) CK(cudaMalloc(&w.nf_cnt.p, sizeof(NFCounters)), "allocating Near-Far counters");
+    w.nf_cap = cap;
+    w.nf_item_bytes = item_bytes;
+    return SSSP_OK;
 }
 
-sssp_status launch_attempt(sssp_graph* g, uint32_t source, unsigned long long* out_dev, cudaStream_t s, int bits) {
-    const unsigned k0 = g->opts.delta_init ? ilog2_round((double)g->opts.delta_init) : heuristic_k(g);
-    sssp_status st = ensure_ring(g, bits == 32 ? 8 : 16, g->cap ? g->cap : default_cap(g));
+template <typename DistT>
+sssp_status launch_nf(sssp_graph* g, Workspace& w, uint32_t source, unsigned long long* out_dev, cudaStream_t s,
+                      int bits, unsigned k0) {
+    const int ib = bits == 32 ? 8 : 16;
+    sssp_status st = ensure_nf(g, w, ib, w.nf_cap ? w.nf_cap : 2 * default_cap(g));
     if (st) return st;
-    if ((st = ensure_trace(g))) return st;
-    if (bits == 32) return launch_one<uint32_t>(g, source, out_dev, s, 32, k0);
-    return launch_one<unsigned long long>(g, source, out_dev, s, 64, k0);
+    void* fn = (void*)near_far_kernel<DistT>;
+    int occ = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, 256, 0), "occupancy query");
+    unsigned grid = (unsigned)(std::max(occ, 1) * g->sm_count);
+    if (g->opts.grid_ctas && g->opts.grid_ctas < grid) grid = g->opts.grid_ctas;
+    NFParams<DistT> p{};
+    p.off = g->d_off;
+    p.adj = g->d_adj;
+    p.dist = (DistT*)w.dist.p;
+    unsigned long long* base = (unsigned long long*)w.nf_piles.p;
+    const size_t words = (size_t)w.nf_cap * (ib / 8);
+    p.near[0] = base;
+    p.near[1] = base + words;
+    p.far[0] = base + 2 * words;
+    p.far[1] = base + 3 * words;
+    p.cnt = (NFCounters*)w.nf_cnt.p;
+    p.ctl = (Ctl*)w.ctl.p;
+    p.cap = w.nf_cap;
+    p.delta = 1ull << std::min(k0, bits == 32 ? 31u : 62u);
+    p.timeout_ns = (unsigned long long)(g->opts.timeout_ms ? g->opts.timeout_ms : 60000u) * 1000000ull;
+    const unsigned aux_grid = (unsigned)g->sm_count * 8;
+    CK(cudaEventRecord(w.ev[0], s), "event");
+    near_far_init_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, g->n, source, p.cnt, p.ctl, p.near[0]);
+    CK(cudaGetLastError(), "init kernel launch");
+    CK(cudaEventRecord(w.ev[1], s), "event");
+    void* args[] = {(void*)&p};
+    CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(256), args, 0, s), "Near-Far kernel launch");
+    CK(cudaEventRecord(w.ev[2], s), "event");
+    finalize_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, out_dev, g->n, g->d_off, p.ctl);
+    CK(cudaGetLastError(), "finalize kernel launch");
+    CK(cudaEventRecord(w.ev[3], s), "event");
+    CK(cudaMemcpyAsync(w.h_ctl, w.ctl.p, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "status copy");
+    w.last_grid = grid;
+    w.last_block = 256;
+    w.last_k0 = std::min(k0, bits == 32 ? 31u : 62u);
+    return SSSP_OK;
 }
 
-void accumulate(sssp_graph* g, const Ctl& c, int bits) {
+sssp_status launch_attempt(sssp_graph* g, Workspace& w, uint32_t source, unsigned long long* out_dev, cudaStream_t s,
+                           int bits, unsigned conc) {
+    if (g->opts.algorithm == SSSP_ALGO_NEAR_FAR) {
+        // static Delta: the Near-Far rule unless given
+        const unsigned k0 = g->opts.delta_init ? ilog2_round((double)g->opts.delta_init) : g->heur_k_nf;
+        if (bits == 32) return launch_nf<uint32_t>(g, w, source, out_dev, s, 32, k0);
+        return launch_nf<unsigned long long>(g, w, source, out_dev, s, 64, k0);
+    }
+    const unsigned k0 = g->opts.delta_init ? ilog2_round((double)g->opts.delta_init) : heuristic_k(g);
+    sssp_status st = ensure_ring(g, w, bits == 32 ? 8 : 16, w.cap ? w.cap : default_cap(g));
+    if (st) return st;
+    if ((st = ensure_trace(g, w))) return st;
+    if (bits == 32) return launch_one<uint32_t>(g, w, source, out_dev, s, 32, k0, conc);
+    return launch_one<unsigned long long>(g, w, source, out_dev, s, 64, k0, conc);
+}
+
+void accumulate(sssp_graph* g, Workspace& w, const Ctl& c, int bits) {
     sssp_stats& st = g->stats;
     st.vertices_processed += c.st_vertices;
     st.edges_relaxed += c.st_edges;
@@ -293,57 +426,75 @@ void accumulate(sssp_graph* g, const Ctl& c, int bits) {
     st.reachable += c.reach_v;
     st.reach_edges += c.reach_e;
     st.max_dist = std::max<uint64_t>(st.max_dist, c.max_dist);
-    st.init_delta_log2 = g->last_k0;
+    st.init_delta_log2 = w.last_k0;
     st.final_delta_log2 = meta_k(c.head.meta);
     st.head_switches += c.head_switches;
     st.delta_changes += c.delta_changes;
     st.dist_bits = (uint32_t)bits;
-    st.grid_ctas = g->last_grid;
-    st.block_threads = g->last_block;
+    st.grid_ctas = w.last_grid;
+    st.block_threads = w.last_block;
     st.runs += 1;
-    st.trace_entries = std::min<uint32_t>(c.trace_count, g->trace_alloc);
+    st.trace_entries = std::min<uint32_t>(c.trace_count, w.trace_alloc);
     float a = 0, b = 0;
-    cudaEventElapsedTime(&a, g->ev[1], g->ev[2]);
-    cudaEventElapsedTime(&b, g->ev[0], g->ev[3]);
+    cudaEventElapsedTime(&a, w.ev[1], w.ev[2]);
+    cudaEventElapsedTime(&b, w.ev[0], w.ev[3]);
     st.kernel_ms += a;
     st.total_ms += b;
 }
 
-// Synchronous run of one source with retry (ring growth / 64-bit distances).
-sssp_status run_one_sync(sssp_graph* g, uint32_t source, unsigned long long* out_dev, cudaStream_t s) {
-    int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
-    for (int attempt = 0; attempt < 24; ++attempt) {
-        sssp_status st = launch_attempt(g, source, out_dev, s, bits);
-        if (st) return st;
-        CK(cudaStreamSynchronize(s), "SSSP run");
-        const unsigned status = g->h_ctl->status;
-        if (status == 0) {
-            accumulate(g, *g->h_ctl, bits);
-            return SSSP_OK;
-        }
-        // aborted attempt: the ring holds leftovers -> clear it before anything else
-        CK(cudaMemsetAsync(g->ring.p, 0xFF, g->ring.bytes, s), "clearing the bucket ring");
-        CK(cudaStreamSynchronize(s), "clearing the bucket ring");
-        if (status & kStTimeout) return fail(SSSP_ERR_TIMEOUT, "device watchdog expired");
-        if (status & kStBug) return fail(SSSP_ERR_CUDA, "internal invariant violated");
-        if (status & kStDistOverflow) {
-            if (g->opts.dist_bits == 32) return fail(SSSP_ERR_INVALID_ARGUMENT, "distances exceed 32 bits (dist_bits=32)");
-            bits = 64;
-            if (!g->opts.dist_bits) g->cur_bits = 64;
-            g->stats.retries += 1;
-            continue;
-        }
-        if (status & kStRingOverflow) {
-            if ((g->opts.flags & SSSP_FLAG_NO_RETRY) || attempt >= 20)
-                return fail(SSSP_ERR_WORKLIST_OVERFLOW, "bucket ring overflow");
-            const unsigned long long ncap = g->cap * 2;
-            g->ring.release();
-            sssp_status st2 = ensure_ring(g, bits == 32 ? 8 : 16, ncap);
+// Inspect a finished attempt.  Returns SSSP_OK and sets *done on success; on a
+// recoverable device status prepares the retry (clears/grows the ring, switches
+// to 64-bit) and leaves *done false; otherwise returns the error.
+sssp_status settle_attempt(sssp_graph* g, Workspace& w, cudaStream_t s, int& bits, int attempt, bool* done) {
+    *done = false;
+    const unsigned status = w.h_ctl->status;
+    if (status == 0) {
+        accumulate(g, w, *w.h_ctl, bits);
+        *done = true;
+        return SSSP_OK;
+    }
+    // aborted attempt: the ring holds leftovers -> clear it before anything else
+    CK(cudaMemsetAsync(w.ring.p, 0xFF, w.ring.bytes, s), "clearing the bucket ring");
+    CK(cudaStreamSynchronize(s), "clearing the bucket ring");
+    if (status & kStTimeout) return fail(SSSP_ERR_TIMEOUT, "device watchdog expired");
+    if (status & kStBug) return fail(SSSP_ERR_CUDA, "internal invariant violated");
+    if (status & kStDistOverflow) {
+        if (g->opts.dist_bits == 32) return fail(SSSP_ERR_INVALID_ARGUMENT, "distances exceed 32 bits (dist_bits=32)");
+        bits = 64;
+        if (!g->opts.dist_bits) g->cur_bits = 64;
+        g->stats.retries += 1;
+        return SSSP_OK;
+    }
+    if (status & kStRingOverflow) {
+        if ((g->opts.flags & SSSP_FLAG_NO_RETRY) || attempt >= 20)
+            return fail(SSSP_ERR_WORKLIST_OVERFLOW, "bucket ring overflow");
+        if (g->opts.algorithm == SSSP_ALGO_NEAR_FAR) {
+            sssp_status st2 = ensure_nf(g, w, w.nf_item_bytes, w.nf_cap * 2);
             if (st2) return st2;
             g->stats.retries += 1;
-            continue;
+            return SSSP_OK;
         }
-        return fail(SSSP_ERR_CUDA, "unknown device status");
+        const unsigned long long ncap = w.cap * 2;
+        w.ring.release();
+        sssp_status st2 = ensure_ring(g, w, bits == 32 ? 8 : 16, ncap);
+        if (st2) return st2;
+        g->stats.retries += 1;
+        return SSSP_OK;
+    }
+    return fail(SSSP_ERR_CUDA, "unknown device status");
+}
+
+// Synchronous run of one source on one workspace, with retry.
+sssp_status run_one_sync(sssp_graph* g, Workspace& w, uint32_t source, unsigned long long* out_dev, cudaStream_t s,
+                         unsigned conc) {
+    int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
+    for (int attempt = 0; attempt < 24; ++attempt) {
+        sssp_status st = launch_attempt(g, w, source, out_dev, s, bits, conc);
+        if (st) return st;
+        CK(cudaStreamSynchronize(s), "SSSP run");
+        bool done = false;
+        if ((st = settle_attempt(g, w, s, bits, attempt, &done))) return st;
+        if (done) return SSSP_OK;
     }
     return fail(SSSP_ERR_WORKLIST_OVERFLOW, "retries exhausted");
 }
@@ -365,6 +516,40 @@ sssp_status classify_out(sssp_graph* g, const void* ptr, bool* is_dev) {
     return SSSP_OK;
 }
 
+// Concurrent batch (device dist_out): groups of c sources, one per workspace
+// and stream; every attempt of a group is launched before any is awaited.
+sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, unsigned long long* out,
+                           cudaStream_t caller, unsigned c) {
+    sssp_status st = ensure_slots(g, c);
+    if (st) return st;
+    CK(cudaEventRecord(g->bev[0], caller), "event");
+    for (unsigned j = 1; j < c; ++j) CK(cudaStreamWaitEvent(g->ws[j]->own_stream, g->bev[0], 0), "stream join");
+    auto slot_stream = [&](unsigned j) { return j == 0 ? caller : g->ws[j]->own_stream; };
+    for (uint32_t i0 = 0; i0 < k && st == SSSP_OK; i0 += c) {
+        const unsigned cnt = std::min<uint32_t>(c, k - i0);
+        int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
+        for (unsigned j = 0; j < cnt && st == SSSP_OK; ++j)
+            st = launch_attempt(g, *g->ws[j], sources[i0 + j], out + (size_t)(i0 + j) * g->n, slot_stream(j), bits, c);
+        for (unsigned j = 0; j < cnt && st == SSSP_OK; ++j) {
+            const cudaError_t e = cudaStreamSynchronize(slot_stream(j));
+            if (e != cudaSuccess) {
+                st = cuda_fail(e, "SSSP run");
+                break;
+            }
+            int b = bits;
+            bool done = false;
+            st = settle_attempt(g, *g->ws[j], slot_stream(j), b, 0, &done);
+            if (st == SSSP_OK && !done)  // recoverable: redo this source alone (still concurrent-sized grid)
+                st = run_one_sync(g, *g->ws[j], sources[i0 + j], out + (size_t)(i0 + j) * g->n, slot_stream(j), c);
+        }
+    }
+    for (unsigned j = 1; j < c; ++j) {
+        cudaEventRecord(g->ws[j]->ev[3], g->ws[j]->own_stream);
+        cudaStreamWaitEvent(caller, g->ws[j]->ev[3], 0);
+    }
+    return st;
+}
+
 sssp_status run_many(sssp_graph* g, const uint32_t* sources, uint32_t k, uint64_t* dist_out, sssp_stream_t stream) {
     if (!g || !dist_out || (k && !sources)) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL argument");
     if (k == 0) return fail(SSSP_ERR_INVALID_ARGUMENT, "k == 0");
@@ -378,6 +563,11 @@ sssp_status run_many(sssp_graph* g, const uint32_t* sources, uint32_t k, uint64_
     cudaStream_t s = (cudaStream_t)stream;
     g->busy = true;
     g->stats = sssp_stats{};
+    Workspace& w0 = *g->ws[0];
+    const unsigned c = g->opts.algorithm == SSSP_ALGO_NEAR_FAR
+                           ? 1u  // grid-wide barriers: one cooperative launch at a time
+                           : std::min<unsigned>(std::max(1u, g->opts.concurrent_sources), k);
+    g->stats.concurrency = (is_dev && c > 1) ? c : 1;
     const bool async = (g->opts.flags & SSSP_FLAG_ASYNC) && is_dev && k == 1;
     if (!is_dev && !g->hostout.p) {
         cudaError_t e = cudaMalloc(&g->hostout.p, (size_t)g->n * 8);
@@ -387,25 +577,37 @@ sssp_status run_many(sssp_graph* g, const uint32_t* sources, uint32_t k, uint64_
         }
         g->hostout.bytes = (size_t)g->n * 8;
     }
-    for (uint32_t i = 0; i < k && st == SSSP_OK; ++i) {
-        unsigned long long* out = is_dev ? (unsigned long long*)dist_out + (size_t)i * g->n
-                                         : (unsigned long long*)g->hostout.p;
-        if (async) {
-            const int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
-            st = launch_attempt(g, sources[i], out, s, bits);
-            if (st == SSSP_OK) {
-                g->async_pending = true;
-                g->stats.dist_bits = (uint32_t)bits;
-            }
-        } else {
-            st = run_one_sync(g, sources[i], out, s);
-            if (st == SSSP_OK && !is_dev) {
-                cudaError_t e = cudaMemcpyAsync((unsigned long long*)dist_out + (size_t)i * g->n, out,
-                                                (size_t)g->n * 8, cudaMemcpyDeviceToHost, s);
-                if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-                if (e != cudaSuccess) st = cuda_fail(e, "copying dist to host");
+    cudaEventRecord(g->bev[0], s);
+    if (is_dev && c > 1) {
+        st = run_concurrent(g, sources, k, (unsigned long long*)dist_out, s, c);
+    } else {
+        for (uint32_t i = 0; i < k && st == SSSP_OK; ++i) {
+            unsigned long long* out = is_dev ? (unsigned long long*)dist_out + (size_t)i * g->n
+                                             : (unsigned long long*)g->hostout.p;
+            if (async) {
+                const int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
+                st = launch_attempt(g, w0, sources[i], out, s, bits, 1);
+                if (st == SSSP_OK) {
+                    g->async_pending = true;
+                    g->stats.dist_bits = (uint32_t)bits;
+                }
+            } else {
+                st = run_one_sync(g, w0, sources[i], out, s, 1);
+                if (st == SSSP_OK && !is_dev) {
+                    cudaError_t e = cudaMemcpyAsync((unsigned long long*)dist_out + (size_t)i * g->n, out,
+                                                    (size_t)g->n * 8, cudaMemcpyDeviceToHost, s);
+                    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+                    if (e != cudaSuccess) st = cuda_fail(e, "copying dist to host");
+                }
             }
         }
+    }
+    cudaEventRecord(g->bev[1], s);
+    if (!async && st == SSSP_OK) {
+        cudaEventSynchronize(g->bev[1]);
+        float ms = 0;
+        cudaEventElapsedTime(&ms, g->bev[0], g->bev[1]);
+        g->stats.batch_ms = ms;
     }
     g->stats.status = st;
     g->busy = false;
@@ -442,6 +644,7 @@ void sssp_options_default(sssp_options* o) {
     o->timeout_ms = 0;
     o->trace_capacity = 0;
     o->active_init = 0;
+    o->concurrent_sources = 1;
 }
 
 sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offsets, const uint32_t* col,
@@ -539,16 +742,8 @@ sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offset
     // they are tried first and the overflow flag triggers a 64-bit re-run.
     g->cur_bits = 32;
 
-    CKG(cudaMalloc(&g->dist.p, (size_t)n * 8), "allocating dist");
-    g->dist.bytes = (size_t)n * 8;
-    CKG(cudaMalloc(&g->expanded.p, ((size_t)n + 31) / 32 * 4), "allocating the expansion bitmap");
-    CKG(cudaMalloc(&g->bk.p, sizeof(BucketCtl) * kMaxBuckets), "allocating bucket counters");
-    CKG(cudaMemset(g->bk.p, 0, sizeof(BucketCtl) * kMaxBuckets), "bucket counters");
-    CKG(cudaMalloc(&g->ctl.p, sizeof(Ctl)), "allocating control block");
-    CKG(cudaMemset(g->ctl.p, 0, sizeof(Ctl)), "control block");
-    CKG(cudaHostAlloc((void**)&g->h_ctl, sizeof(Ctl), cudaHostAllocDefault), "allocating pinned status block");
-    for (auto& e : g->ev) CKG(cudaEventCreate(&e), "creating events");
-    sssp_status st2 = ensure_ring(g, (o.dist_bits == 64) ? 16 : 8, default_cap(g));
+    for (auto& e : g->bev) CKG(cudaEventCreate(&e), "creating events");
+    sssp_status st2 = ensure_slots(g, 1);
     if (st2) return bail(st2);
 #undef CKG
     *out = g;
@@ -561,16 +756,14 @@ sssp_status sssp_graph_destroy(sssp_graph* g) {
     cudaDeviceSynchronize();
     if (g->d_off) cudaFree(g->d_off);
     if (g->d_adj) cudaFree(g->d_adj);
-    g->dist.release();
-    g->ring.release();
-    g->bk.release();
-    g->ctl.release();
-    g->trace.release();
+    for (Workspace* w : g->ws) {
+        w->release();
+        delete w;
+    }
+    g->ws.clear();
     g->scratch.release();
-    g->expanded.release();
     g->hostout.release();
-    if (g->h_ctl) cudaFreeHost(g->h_ctl);
-    for (auto& e : g->ev)
+    for (auto& e : g->bev)
         if (e) cudaEventDestroy(e);
     delete g;
     return SSSP_OK;
@@ -588,8 +781,10 @@ sssp_status sssp_set_options(sssp_graph* g, const sssp_options* opts) {
     if (opts->dist_bits) g->cur_bits = (int)opts->dist_bits;
     else g->cur_bits = 32;
     if (ring_change) {
-        g->ring.release();
-        g->cap = 0;
+        for (Workspace* w : g->ws) {
+            w->ring.release();
+            w->cap = 0;
+        }
     }
     return SSSP_OK;
 }
@@ -608,14 +803,15 @@ sssp_status sssp_get_stats(sssp_graph* g, sssp_stats* out) {
     if (g->async_pending) {
         DeviceGuard dg(g->device);
         g->async_pending = false;
-        cudaError_t e = cudaEventSynchronize(g->ev[3]);
+        Workspace& w = *g->ws[0];
+        cudaError_t e = cudaEventSynchronize(w.ev[3]);
         if (e != cudaSuccess) return cuda_fail(e, "async run");
         // the status copy was enqueued after ev[3] on the same stream
         e = cudaDeviceSynchronize();
         if (e != cudaSuccess) return cuda_fail(e, "async run");
-        const unsigned status = g->h_ctl->status;
+        const unsigned status = w.h_ctl->status;
         if (status) {
-            cudaMemset(g->ring.p, 0xFF, g->ring.bytes);
+            cudaMemset(w.ring.p, 0xFF, w.ring.bytes);
             cudaDeviceSynchronize();
             g->stats.status = (status & kStRingOverflow)   ? SSSP_ERR_WORKLIST_OVERFLOW
                               : (status & kStTimeout)      ? SSSP_ERR_TIMEOUT
@@ -624,7 +820,7 @@ sssp_status sssp_get_stats(sssp_graph* g, sssp_stats* out) {
             *out = g->stats;
             return fail((sssp_status)g->stats.status, "async run failed (status bits " + std::to_string(status) + ")");
         }
-        accumulate(g, *g->h_ctl, (int)g->stats.dist_bits);
+        accumulate(g, w, *w.h_ctl, (int)g->stats.dist_bits);
         g->stats.status = SSSP_OK;
     }
     *out = g->stats;
@@ -634,12 +830,13 @@ sssp_status sssp_get_stats(sssp_graph* g, sssp_stats* out) {
 sssp_status sssp_get_trace(sssp_graph* g, sssp_trace_entry* out, uint32_t cap, uint32_t* count) {
     if (!g || !count || (cap && !out)) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL argument");
     *count = 0;
-    if (!g->trace.p) return SSSP_OK;
-    const uint32_t nvalid = std::min<uint32_t>(g->stats.trace_entries, g->trace_alloc);
+    Workspace& w = *g->ws[0];
+    if (!w.trace.p) return SSSP_OK;
+    const uint32_t nvalid = std::min<uint32_t>(g->stats.trace_entries, w.trace_alloc);
     const uint32_t c = std::min(cap, nvalid);
     if (c) {
         DeviceGuard dg(g->device);
-        CK(cudaMemcpy(out, g->trace.p, (size_t)c * sizeof(sssp_trace_entry), cudaMemcpyDeviceToHost), "trace copy");
+        CK(cudaMemcpy(out, w.trace.p, (size_t)c * sizeof(sssp_trace_entry), cudaMemcpyDeviceToHost), "trace copy");
     }
     *count = c;
     return SSSP_OK;
@@ -648,7 +845,8 @@ sssp_status sssp_get_trace(sssp_graph* g, sssp_trace_entry* out, uint32_t cap, u
 sssp_status sssp_get_profile(sssp_graph* g, uint64_t* out, uint32_t cap, uint32_t* count) {
     if (!g || !count || (cap && !out)) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL argument");
     const uint32_t c = std::min<uint32_t>(cap, kProfCounters);
-    for (uint32_t i = 0; i < c; ++i) out[i] = g->h_ctl ? g->h_ctl->prof[i] : 0;
+    const Ctl* hc = g->ws.empty() ? nullptr : g->ws[0]->h_ctl;
+    for (uint32_t i = 0; i < c; ++i) out[i] = hc ? hc->prof[i] : 0;
     *count = c;
     return SSSP_OK;
 }

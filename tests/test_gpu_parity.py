@@ -105,6 +105,9 @@ PERTURB = [
     dict(ring_items=64), dict(ring_items=256, num_buckets=4),
     dict(flags=sssp.SSSP_FLAG_TRACE),
     dict(flags=sssp.SSSP_FLAG_NO_LOCAL), dict(local_max=1), dict(local_max=16), dict(max_backoff_ns=64),
+    dict(algorithm=sssp.SSSP_ALGO_NEAR_FAR), dict(algorithm=sssp.SSSP_ALGO_NEAR_FAR, delta_init=1),
+    dict(algorithm=sssp.SSSP_ALGO_NEAR_FAR, delta_init=1 << 40), dict(algorithm=sssp.SSSP_ALGO_NEAR_FAR, ring_items=64),
+    dict(algorithm=sssp.SSSP_ALGO_NEAR_FAR, grid_ctas=5), dict(flags=sssp.SSSP_FLAG_ADAPT_ACTIVE),
 ]
 
 
@@ -252,3 +255,47 @@ def test_loaded_file_through_the_abi(tmp_path):
     h = loaders.load(p)
     s = int(gg.config_sources("road", h, 1)[0])
     check(h, s)
+
+
+@pytest.mark.parametrize("conc", [2, 3, 8])
+def test_concurrent_batch(conc):
+    """NEXT-1: several sources in flight at once (own workspace + stream each)."""
+    g = gg.make("rmat", scale_down=9)
+    srcs = gg.sources(g, 7, seed=5)
+    G = sssp.Graph.from_csr(g, concurrent_sources=conc)
+    D = G.run_batch(srcs)
+    st = G.stats()
+    assert st["runs"] == 7 and st["concurrency"] == min(conc, 7) and st["batch_ms"] > 0
+    for i, s in enumerate(srcs):
+        assert np.array_equal(sssp.to_u64(D[i]), oracle.dijkstra(g, int(s))[0])
+
+
+def test_concurrent_batch_with_overflow_retry():
+    g = gg.make("road", scale_down=8)
+    srcs = gg.config_sources("road", g, 4)
+    G = sssp.Graph.from_csr(g, concurrent_sources=4, ring_items=64)
+    D = G.run_batch(srcs)
+    assert G.stats()["retries"] >= 1
+    for i, s in enumerate(srcs):
+        assert np.array_equal(sssp.to_u64(D[i]), oracle.dijkstra(g, int(s))[0])
+
+
+@pytest.mark.parametrize("config", ["road", "rmat", "er"])
+def test_near_far_ablation_full_size(config):
+    """NEXT-2: the BSP Near-Far comparison system gives the same bits."""
+    g = gg.make(config, scale_down=4)
+    s = int(gg.config_sources(config, g, 1)[0])
+    st = check(g, s, algorithm=sssp.SSSP_ALGO_NEAR_FAR)
+    assert st["head_switches"] > 0  # supersteps
+
+
+def test_near_far_u64_and_golden():
+    n = 10
+    g = gg.from_arcs(n, [(i, i + 1, 0xFFFFFFFF) for i in range(n - 1)] + [(0, 5, 7)])
+    st = check(g, 0, algorithm=sssp.SSSP_ALGO_NEAR_FAR)
+    assert st["dist_bits"] == 64
+    for name in golden_names():
+        fx = load_golden(name)
+        gg2 = gg.from_arcs(fx["n"], fx["arcs"])
+        d, _ = gpu_dist(gg2, fx["source"], algorithm=sssp.SSSP_ALGO_NEAR_FAR)
+        assert [int(x) for x in d] == fx["dist"]
