@@ -182,7 +182,10 @@ def run_ours(args, world, rank, local):
         n_src = len(srcs)
     else:
         srcs = step_sources(args.config, g, world, rank, n_src)
-    G = sssp.Graph.from_csr(g, device=local)
+    opts = dict(device=local, algorithm=sssp.SSSP_ALGO_NEAR_FAR if args.algorithm == "nearfar" else sssp.SSSP_ALGO_ADDS)
+    if args.config == "batch":
+        opts["concurrent_sources"] = args.concurrency
+    G = sssp.Graph.from_csr(g, **opts)
     stream = torch.cuda.current_stream(dev)
     out = torch.empty(g.n, dtype=torch.int64, device=dev)
 
@@ -301,7 +304,9 @@ def run_ours(args, world, rank, local):
                        "parallelism": f"source-partitioned x{world} (graph replicated)",
                        "l2": f"inputs larger than L2 (CSR {csr_bytes / 2**20:.0f} MiB > 126 MiB), no flush"
                        if csr_bytes > L2_BYTES else "small input (L2-resident)",
-                       "grid_ctas": last["grid_ctas"], "block_threads": last["block_threads"]},
+                       "grid_ctas": last["grid_ctas"], "block_threads": last["block_threads"],
+                       "algorithm": args.algorithm,
+                       "concurrent_sources": (args.concurrency if args.config == "batch" else 1)},
             "ms_per_source": T / units,
             "work_efficiency": {"edges": Eg_all / max(1, E_all), "vertices": Vg_all / max(1, V_all)},
             "delta_log2": {"init": last["init_delta_log2"], "final": last["final_delta_log2"]},
@@ -331,6 +336,9 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--algorithm", default="adds", choices=["adds", "nearfar"],
+                    help="nearfar = the paper's BSP comparison system (ablation, NEXT-2)")
+    ap.add_argument("--concurrency", type=int, default=4, help="sources in flight per GPU for --config batch")
     args = ap.parse_args()
     world, rank, local = dist_init()
     if args.impl == "reference":

@@ -427,7 +427,7 @@ void accumulate(sssp_graph* g, Workspace& w, const Ctl& c, int bits) {
     st.reach_edges += c.reach_e;
     st.max_dist = std::max<uint64_t>(st.max_dist, c.max_dist);
     st.init_delta_log2 = w.last_k0;
-    st.final_delta_log2 = meta_k(c.head.meta);
+    st.final_delta_log2 = g->opts.algorithm == SSSP_ALGO_NEAR_FAR ? w.last_k0 : meta_k(c.head.meta);
     st.head_switches += c.head_switches;
     st.delta_changes += c.delta_changes;
     st.dist_bits = (uint32_t)bits;
