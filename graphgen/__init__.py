@@ -64,6 +64,8 @@ def _L():
         lib.gg_hash.restype = u64
         lib.gg_hash.argtypes = [u64, u64, u64]
         lib.gg_num_threads.restype = ctypes.c_int
+        lib.gg_float_weights.restype = None
+        lib.gg_float_weights.argtypes = [u64, ctypes.c_float, ctypes.c_float, u64, p]
         _lib = lib
     return _lib
 
@@ -150,6 +152,13 @@ def sources(g: CSR, k: int, seed: int) -> np.ndarray:
     out = np.empty(max(k, 1), dtype=np.uint32)
     got = _L().gg_sources(g.n, _ptr(g.row_offsets), seed, k, _ptr(out), (1 << 20) + 64 * k)
     return out[:got].copy()
+
+
+def float_weights(g: CSR, lo: float, hi: float, seed: int) -> np.ndarray:
+    """float32 arc weights in [lo, hi) for graph g (NEXT-3), seeded and thread-count independent."""
+    w = np.empty(max(g.m, 1), dtype=np.float32)[:g.m]
+    _L().gg_float_weights(g.m, lo, hi, seed, _ptr(w))
+    return w
 
 
 def gg_hash(seed: int, stream: int, i: int) -> int:

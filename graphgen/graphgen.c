@@ -49,7 +49,7 @@ uint64_t gg_hash(uint64_t seed, uint64_t stream, uint64_t i) {
 }
 
 enum { ST_GRID_W = 1, ST_RMAT_LVL = 2, ST_RMAT_PERM = 3, ST_RMAT_W = 4,
-       ST_ER_EP = 5, ST_ER_W = 6, ST_SRC = 7 };
+       ST_ER_EP = 5, ST_ER_W = 6, ST_SRC = 7, ST_FLOAT_W = 8 };
 
 /* ------------------------------------------------------------------ grid */
 /* number of arcs of a W x H 4-neighbour lattice */
@@ -245,4 +245,16 @@ int gg_num_threads(void) {
 #else
     return 1;
 #endif
+}
+
+/* float32 weights for an existing CSR (NEXT-3): w = lo + u * (hi - lo) with u a
+ * 24-bit uniform in [0, 1) from the counter RNG (exactly representable), rounded
+ * to binary32; independent of the integer weights. */
+void gg_float_weights(uint64_t m, float lo, float hi, uint64_t seed, float *w) {
+    uint64_t key = gg_key(seed, ST_FLOAT_W);
+#pragma omp parallel for schedule(static)
+    for (int64_t e = 0; e < (int64_t)m; ++e) {
+        float u = (float)(gg_draw(key, (uint64_t)e) >> 40) * (1.0f / 16777216.0f);
+        w[e] = lo + u * (hi - lo);
+    }
 }

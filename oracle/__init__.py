@@ -9,6 +9,7 @@ passages each function follows).
 Functions
 ---------
 dijkstra(g, s)        -> (dist uint64[n], V_dij, E_dij)   binary-heap Dijkstra
+dijkstra_f32(g, wf, s)-> float32 distances with IEEE-rounded path sums (NEXT-3)
 certify(g, s, dist)   -> 0 if dist is exact, else clause code
 reach_counts(g, dist) -> (V, E) recomputed from a distance vector
 """
@@ -47,6 +48,8 @@ def _L():
         lib.oracle_dijkstra.argtypes = [u64, u64, p, p, p, u32, p, p, p]
         lib.oracle_certify.restype = ctypes.c_int
         lib.oracle_certify.argtypes = [u64, u64, p, p, p, u32, p, p]
+        lib.oracle_dijkstra_f32.restype = ctypes.c_int
+        lib.oracle_dijkstra_f32.argtypes = [u64, u64, p, p, p, u32, p, p, p]
         lib.oracle_reach_counts.restype = None
         lib.oracle_reach_counts.argtypes = [u64, p, p, p, p]
         _lib = lib
@@ -71,6 +74,22 @@ def dijkstra(g, s: int):
                               dist.ctypes.data, ctypes.byref(V), ctypes.byref(E))
     if rc != 0:
         raise ValueError(f"oracle_dijkstra failed (rc={rc})")
+    return dist, int(V.value), int(E.value)
+
+
+def dijkstra_f32(g, wf, s: int):
+    """Float32-weight SSSP (NEXT-3): dist[v] = min over paths of the float-rounded
+    left-to-right path sum; +inf when unreachable.  ``wf`` = float32[m] weights."""
+    off, col, _ = _arrays(g)
+    w = np.ascontiguousarray(wf, dtype=np.float32)
+    n = len(off) - 1
+    dist = np.empty(n, dtype=np.float32)
+    V = ctypes.c_uint64(0)
+    E = ctypes.c_uint64(0)
+    rc = _L().oracle_dijkstra_f32(n, len(col), off.ctypes.data, col.ctypes.data, w.ctypes.data, int(s),
+                                  dist.ctypes.data, ctypes.byref(V), ctypes.byref(E))
+    if rc != 0:
+        raise ValueError(f"oracle_dijkstra_f32 failed (rc={rc})")
     return dist, int(V.value), int(E.value)
 
 

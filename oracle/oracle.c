@@ -156,3 +156,76 @@ void oracle_reach_counts(uint64_t n, const uint64_t *off, const uint64_t *dist,
         if (dist[v] != INF) { V += 1; E += off[v + 1] - off[v]; }
     *V_out = V; *E_out = E;
 }
+
+/* ---------------------------------------------------------------- float32 weights (NEXT-3)
+ * The paper's float variant: non-negative float weights, distances
+ * accumulated in float.  What is computed (reading R16 in DESIGN.md): the same
+ * refinement dist[v] = min(dist[v], fl(dist[u] + w)) with fl = IEEE binary32
+ * round-to-nearest-even addition, from dist[s] = 0, all others +infinity.
+ * Since fl(x + w) >= x for w >= 0 and fl is monotone, Dijkstra's order is still
+ * valid and the result is the minimum over paths of the left-to-right
+ * float-rounded path sum.  Unreachable (or overflowing to +inf) = +inf. */
+typedef struct { float d; uint32_t v; } fitem_t;
+typedef struct { fitem_t *a; uint64_t size, cap; } fheap_t;
+
+static int fheap_push(fheap_t *h, float d, uint32_t v) {
+    if (h->size == h->cap) {
+        uint64_t nc = h->cap ? 2 * h->cap : 1024;
+        fitem_t *na = (fitem_t *)realloc(h->a, nc * sizeof(fitem_t));
+        if (!na) return -1;
+        h->a = na; h->cap = nc;
+    }
+    uint64_t i = h->size++;
+    while (i > 0) {
+        uint64_t p = (i - 1) / 2;
+        if (h->a[p].d <= d) break;
+        h->a[i] = h->a[p]; i = p;
+    }
+    h->a[i].d = d; h->a[i].v = v;
+    return 0;
+}
+
+static fitem_t fheap_pop(fheap_t *h) {
+    fitem_t top = h->a[0];
+    fitem_t last = h->a[--h->size];
+    uint64_t i = 0, n = h->size;
+    for (;;) {
+        uint64_t l = 2 * i + 1, r = l + 1, c = l;
+        if (l >= n) break;
+        if (r < n && h->a[r].d < h->a[l].d) c = r;
+        if (h->a[c].d >= last.d) break;
+        h->a[i] = h->a[c]; i = c;
+    }
+    if (n) h->a[i] = last;
+    return top;
+}
+
+int oracle_dijkstra_f32(uint64_t n, uint64_t m, const uint64_t *off, const uint32_t *col,
+                        const float *w, uint32_t s, float *dist_out, uint64_t *V_out, uint64_t *E_out) {
+    (void)m;
+    if (s >= n) return -1;
+    const float inf = __builtin_inff();
+    for (uint64_t v = 0; v < n; ++v) dist_out[v] = inf;
+    fheap_t h = { 0, 0, 0 };
+    uint64_t V = 0, E = 0;
+    dist_out[s] = 0.0f;
+    if (fheap_push(&h, 0.0f, s)) return -1;
+    while (h.size) {
+        fitem_t it = fheap_pop(&h);
+        uint32_t u = it.v;
+        if (it.d > dist_out[u]) continue;
+        V += 1;
+        E += off[u + 1] - off[u];
+        for (uint64_t e = off[u]; e < off[u + 1]; ++e) {
+            volatile float nd = it.d + w[e];  /* binary32 RN addition (SSE, no excess precision) */
+            if (nd < dist_out[col[e]]) {
+                dist_out[col[e]] = nd;
+                if (fheap_push(&h, nd, col[e])) { free(h.a); return -1; }
+            }
+        }
+    }
+    free(h.a);
+    if (V_out) *V_out = V;
+    if (E_out) *E_out = E;
+    return 0;
+}
