@@ -146,7 +146,7 @@ typedef struct sssp_stats {
     uint64_t stale_skips;        /* popped items whose distance was already improved */
     uint64_t reachable;          /* vertices with finite distance  (= V_dij) */
     uint64_t reach_edges;        /* sum of out-degrees of reachable vertices (= E_dij, GTEPS numerator) */
-    uint64_t max_dist;           /* largest finite distance */
+    uint64_t max_dist;           /* largest finite distance (float32 graphs: its IEEE bit pattern) */
     uint32_t init_delta_log2;    /* log2 of the initial Delta */
     uint32_t final_delta_log2;   /* log2 of Delta when the run ended */
     uint32_t head_switches;      /* head-bucket advances */
@@ -200,6 +200,17 @@ sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t *row_offset
                               const uint32_t *col, const uint32_t *w,
                               const sssp_options *opts, sssp_graph **out);
 
+/* Float32 weights (NEXT-3; the paper's float variant): w[m] are
+ * non-negative IEEE binary32 values (-0.0 is folded into +0.0; a negative or NaN
+ * weight is SSSP_ERR_INVALID_GRAPH with the first bad index; +inf arcs never
+ * improve anything).  Distances are accumulated in binary32 with
+ * round-to-nearest-even addition: dist[v] = min over paths of the left-to-right
+ * float-rounded path sum (bit-exactly what a float Dijkstra computes).  Such a
+ * handle is run with sssp_run_f32 / sssp_run_batch_f32 only. */
+sssp_status sssp_graph_create_f32(uint32_t n, uint64_t m, const uint64_t *row_offsets,
+                                  const uint32_t *col, const float *w,
+                                  const sssp_options *opts, sssp_graph **out);
+
 /* Releases everything the handle owns (synchronises its device first). NULL-safe. */
 sssp_status sssp_graph_destroy(sssp_graph *g);
 
@@ -225,6 +236,13 @@ sssp_status sssp_run(sssp_graph *g, uint32_t source, uint64_t *dist_out, sssp_st
  * INVALID_ARGUMENT for k == 0 or any source >= n (checked before any work). */
 sssp_status sssp_run_batch(sssp_graph *g, const uint32_t *sources, uint32_t k,
                            uint64_t *dist_out, sssp_stream_t stream);
+
+/* Float32-weight runs: dist_out[v] (float, n entries; k*n for the batch), +inf
+ * when unreachable.  Same stream / error semantics as sssp_run(_batch);
+ * INVALID_ARGUMENT when the handle was created with integer weights. */
+sssp_status sssp_run_f32(sssp_graph *g, uint32_t source, float *dist_out, sssp_stream_t stream);
+sssp_status sssp_run_batch_f32(sssp_graph *g, const uint32_t *sources, uint32_t k,
+                               float *dist_out, sssp_stream_t stream);
 
 /* Statistics of the last run/batch (valid after the run's stream is
  * synchronised).  With SSSP_FLAG_ASYNC this also performs the deferred

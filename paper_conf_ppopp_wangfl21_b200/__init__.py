@@ -103,10 +103,14 @@ SIGNATURES = [
     ("sssp_options_default", None, [ctypes.POINTER(sssp_options)]),
     ("sssp_graph_create", ctypes.c_int,
      [ctypes.c_uint32, ctypes.c_uint64, _P, _P, _P, ctypes.POINTER(sssp_options), ctypes.POINTER(_P)]),
+    ("sssp_graph_create_f32", ctypes.c_int,
+     [ctypes.c_uint32, ctypes.c_uint64, _P, _P, _P, ctypes.POINTER(sssp_options), ctypes.POINTER(_P)]),
     ("sssp_graph_destroy", ctypes.c_int, [_P]),
     ("sssp_set_options", ctypes.c_int, [_P, ctypes.POINTER(sssp_options)]),
     ("sssp_run", ctypes.c_int, [_P, ctypes.c_uint32, _P, _P]),
     ("sssp_run_batch", ctypes.c_int, [_P, _P, ctypes.c_uint32, _P, _P]),
+    ("sssp_run_f32", ctypes.c_int, [_P, ctypes.c_uint32, _P, _P]),
+    ("sssp_run_batch_f32", ctypes.c_int, [_P, _P, ctypes.c_uint32, _P, _P]),
     ("sssp_get_stats", ctypes.c_int, [_P, ctypes.POINTER(sssp_stats)]),
     ("sssp_get_trace", ctypes.c_int, [_P, _P, ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint32)]),
     ("sssp_get_profile", ctypes.c_int, [_P, _P, ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint32)]),
@@ -175,6 +179,16 @@ def _as_host_or_dev(a, dtype):
     return arr.ctypes.data, arr
 
 
+def _is_float(a) -> bool:
+    try:
+        import torch
+        if isinstance(a, torch.Tensor):
+            return a.dtype == torch.float32
+    except ImportError:  # pragma: no cover
+        pass
+    return np.asarray(a).dtype == np.float32
+
+
 def _stream_ptr(stream):
     if stream is None:
         import torch
@@ -195,15 +209,18 @@ class Graph:
         self.options = options
         self.n = int(len(row_offsets) - 1)
         self.m = int(len(col))
+        self.f32 = _is_float(w)
         po, k1 = _as_host_or_dev(row_offsets, np.uint64)
         pc, k2 = _as_host_or_dev(col, np.uint32)
-        pw, k3 = _as_host_or_dev(w, np.uint32)
-        _check(L.sssp_graph_create(self.n, self.m, po, pc, pw, ctypes.byref(options), ctypes.byref(self._h)))
+        pw, k3 = _as_host_or_dev(w, np.float32 if self.f32 else np.uint32)
+        create = L.sssp_graph_create_f32 if self.f32 else L.sssp_graph_create
+        _check(create(self.n, self.m, po, pc, pw, ctypes.byref(options), ctypes.byref(self._h)))
         self.device = options.device
 
     @classmethod
-    def from_csr(cls, csr, **kw):
-        return cls(csr.row_offsets, csr.col, csr.w, **kw)
+    def from_csr(cls, csr, weights=None, **kw):
+        """``weights`` overrides csr.w (e.g. float32 weights from graphgen.float_weights)."""
+        return cls(csr.row_offsets, csr.col, csr.w if weights is None else weights, **kw)
 
     def close(self):
         if getattr(self, "_h", None) and self._h.value:
@@ -227,18 +244,21 @@ class Graph:
         self.options = o
 
     def run(self, source: int, out=None, stream=None):
-        """dist[v] from ``source`` as a torch.int64 cuda tensor (UINT64_MAX reads as -1)."""
+        """dist[v] from ``source`` as a cuda tensor: torch.int64 (UINT64_MAX reads as -1) for
+        integer weights, torch.float32 (+inf when unreachable) for float32 weights."""
         import torch
         if out is None:
-            out = torch.empty(self.n, dtype=torch.int64, device=f"cuda:{self.device}")
-        _check(lib().sssp_run(self._h, int(source), out.data_ptr(), _stream_ptr(stream)))
+            out = torch.empty(self.n, dtype=torch.float32 if self.f32 else torch.int64, device=f"cuda:{self.device}")
+        fn = lib().sssp_run_f32 if self.f32 else lib().sssp_run
+        _check(fn(self._h, int(source), out.data_ptr(), _stream_ptr(stream)))
         return out
 
     def run_host(self, source: int, out: np.ndarray | None = None, stream=None) -> np.ndarray:
         """Same, into host memory (the library copies the result back)."""
         if out is None:
-            out = np.empty(self.n, dtype=np.uint64)
-        _check(lib().sssp_run(self._h, int(source), out.ctypes.data, _stream_ptr(stream)))
+            out = np.empty(self.n, dtype=np.float32 if self.f32 else np.uint64)
+        fn = lib().sssp_run_f32 if self.f32 else lib().sssp_run
+        _check(fn(self._h, int(source), out.ctypes.data, _stream_ptr(stream)))
         return out
 
     def run_batch(self, sources, out=None, stream=None):
@@ -246,8 +266,10 @@ class Graph:
         import torch
         src = np.ascontiguousarray(sources, dtype=np.uint32)
         if out is None:
-            out = torch.empty((len(src), self.n), dtype=torch.int64, device=f"cuda:{self.device}")
-        _check(lib().sssp_run_batch(self._h, src.ctypes.data, len(src), out.data_ptr(), _stream_ptr(stream)))
+            out = torch.empty((len(src), self.n), dtype=torch.float32 if self.f32 else torch.int64,
+                              device=f"cuda:{self.device}")
+        fn = lib().sssp_run_batch_f32 if self.f32 else lib().sssp_run_batch
+        _check(fn(self._h, src.ctypes.data, len(src), out.data_ptr(), _stream_ptr(stream)))
         return out
 
     def stats(self) -> dict:

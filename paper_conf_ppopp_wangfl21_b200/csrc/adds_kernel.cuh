@@ -300,6 +300,40 @@ __device__ void periodic_step(const Params<DistT>& p, const int lane) {
     commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 2u, d.flags);
 }
 
+// --------------------------------------------------------------- weight arithmetic
+// Integer weights: nd = d + w in 64 bits, Delta = 2^k, bucket = nd >> k.
+// Float32 weights (NEXT-3): d and w are IEEE binary32 bit patterns (non-negative
+// floats order like their bits, so dist keeps the native u32 atomicMin);
+// nd = fl(d + w) round-to-nearest; Delta = 2^(k - kFloatBias), k biased so that
+// Delta can be below 1.
+constexpr int kFloatBias = 64;
+template <bool kF>
+__device__ __forceinline__ unsigned long long relax_sum(unsigned long long d, unsigned w) {
+    if constexpr (kF)
+        return (unsigned long long)__float_as_uint(__fadd_rn(__uint_as_float((unsigned)d), __uint_as_float(w)));
+    else
+        return d + w;
+}
+// a sum that can never be an improvement (float: +inf / NaN) or that overflows
+// the distance type (integer: re-run with 64-bit distances)
+template <bool kF>
+__device__ __forceinline__ bool sum_unusable(unsigned long long nd, unsigned long long inf) {
+    if constexpr (kF) return nd >= 0x7F800000ull;
+    else return nd >= inf;
+}
+template <bool kF>
+__device__ __forceinline__ unsigned bucket_of(unsigned long long nd, unsigned k, unsigned long long h, unsigned nb) {
+    if constexpr (kF) {
+        const float jf = __uint_as_float((unsigned)nd) * ldexpf(1.0f, kFloatBias - (int)k);  // exact scaling
+        const unsigned long long j = jf >= 4.0e18f ? (1ull << 62) : (unsigned long long)jf;
+        if (j <= h) return 0u;
+        const unsigned long long o = j - h;
+        return o >= (unsigned long long)(nb - 1) ? nb - 1 : (unsigned)o;
+    } else {
+        return adds_bucket_offset(nd, k, h, nb);
+    }
+}
+
 // --------------------------------------------------------------- shared memory
 constexpr size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
 
@@ -321,7 +355,7 @@ struct Smem {
 };
 
 // --------------------------------------------------------------- kernel
-template <typename DistT, int BT, int EPT, int W>
+template <typename DistT, int BT, int EPT, int W, bool kF>
 __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Params<DistT> p) {
     using IT = ItemT<DistT>;
     using Raw = typename IT::Raw;
@@ -648,7 +682,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                         const unsigned q = j * BT + tid;
                         if (q < Ew) {
                             a[j] = ld_stream_u2(p.adj + s_ebeg[own[j]] + (q - s_scan[own[j]]), pol_stream);
-                            nd[j] = (unsigned long long)s_d[own[j]] + a[j].y;
+                            nd[j] = relax_sum<kF>((unsigned long long)s_d[own[j]], a[j].y);
                             cur[j] = DistInf<DistT>::value;  // tiny batch: straight to atomicMin
                         } else {
                             a[j] = make_uint2(0u, 0u);
@@ -667,7 +701,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                         const unsigned q = rbase + j * BT + tid;
                         if (q < Ew) {
                             a[j] = s_arc[q];
-                            nd[j] = (unsigned long long)s_d[s_owner[q]] + a[j].y;
+                            nd[j] = relax_sum<kF>((unsigned long long)s_d[s_owner[q]], a[j].y);
                         } else {
                             a[j] = make_uint2(0u, 0u);
                             nd[j] = kInf;
@@ -682,8 +716,8 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                     const unsigned q = rbase + j * BT + tid;
                     push[j] = false;
                     if (q < Ew) {
-                        if (nd[j] >= kInf) {
-                            atomicOr(&p.ctl->status, kStDistOverflow);  // 32-bit distances insufficient
+                        if (sum_unusable<kF>(nd[j], kInf)) {
+                            if (!kF) atomicOr(&p.ctl->status, kStDistOverflow);  // 32-bit distances insufficient
                         } else if (nd[j] < (unsigned long long)cur[j]) {
                             const DistT old = atomic_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
                             push[j] = nd[j] < (unsigned long long)old;
@@ -693,7 +727,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {
                     if (!__any_sync(FULL, push[j])) continue;
-                    const unsigned o = push[j] ? adds_bucket_offset(nd[j], k, hd.h, p.nb) : 0u;
+                    const unsigned o = push[j] ? bucket_of<kF>(nd[j], k, hd.h, p.nb) : 0u;
                     // head-bucket children stay in this CTA (warp-aggregated slot grab)
                     bool kept = false;
                     if (lcap) {

@@ -110,4 +110,51 @@ __global__ void finalize_kernel(const DistT* __restrict__ dist, unsigned long lo
     }
 }
 
+// float32-weight graphs (NEXT-3): validate (no negative or NaN weight), fold
+// -0.0 into +0.0 (bit order must equal value order), interleave, max weight
+__global__ void interleave_f32_kernel(const unsigned* __restrict__ col, unsigned* __restrict__ wbits,
+                                      uint2* __restrict__ adj, unsigned long long m, unsigned long long* bad_w,
+                                      unsigned* max_w) {
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    unsigned mx = 0;
+    for (unsigned long long e = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; e < m; e += stride) {
+        unsigned wb = wbits[e];
+        if (wb == 0x80000000u) wb = 0u;                       // -0.0 -> +0.0
+        if ((wb & 0x80000000u) || (wb & 0x7FFFFFFFu) > 0x7F800000u) atomicMin(bad_w, e);  // negative / NaN
+        adj[e] = make_uint2(col[e], wb);
+        if (wb <= 0x7F800000u) mx = wb > mx ? wb : mx;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    if ((threadIdx.x & 31) == 0) atomicMax(max_w, mx);
+}
+
+__global__ void finalize_f32_kernel(const unsigned* __restrict__ dist, float* __restrict__ out, unsigned n,
+                                    const unsigned long long* __restrict__ off, Ctl* ctl) {
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    unsigned long long rv = 0, re = 0, mx = 0;
+    for (unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
+        const unsigned d = dist[v];
+        if (d >= 0x7F800000u) {  // never reached (internal sentinel) or +inf
+            out[v] = __uint_as_float(0x7F800000u);
+        } else {
+            out[v] = __uint_as_float(d);
+            rv += 1;
+            re += off[v + 1] - off[v];
+            mx = d > mx ? d : mx;
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        rv += __shfl_xor_sync(0xffffffffu, rv, o);
+        re += __shfl_xor_sync(0xffffffffu, re, o);
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    }
+    if ((threadIdx.x & 31) == 0 && rv) {
+        atomicAdd(&ctl->reach_v, rv);
+        atomicAdd(&ctl->reach_e, re);
+        atomicMax(&ctl->max_dist, mx);
+    }
+}
+
 }  // namespace adds

@@ -110,6 +110,7 @@ struct sssp_graph {
     uint32_t heur_k_span = 0;  // log2 initial Delta, max_w / B rule (ring span)
     uint32_t heur_k_md = 0;    // log2 initial Delta, max_w / D rule
     uint32_t heur_k_nf = 0;    // log2 initial Delta, Near-Far C*W/D rule
+    bool f32 = false;          // float32 weights (NEXT-3): max_w holds the IEEE bits
     sssp_options opts{};
     int sm_count = 0;
     std::vector<Workspace*> ws;
@@ -161,12 +162,13 @@ struct KVariant {
     void* fn;
     size_t smem;
 };
-template <typename DistT, int BT>
+template <typename DistT, int BT, bool kF = false>
 KVariant kvar() {
     constexpr int W = BT >= 1024 ? 4096 : (BT >= 256 ? 2048 : 1024);
-    return KVariant{(void*)adds_persistent_kernel<DistT, BT, 4, W>, Smem<DistT, BT, 4, W>::bytes};
+    return KVariant{(void*)adds_persistent_kernel<DistT, BT, 4, W, kF>, Smem<DistT, BT, 4, W>::bytes};
 }
-KVariant persistent_variant(int bits, int bt) {
+KVariant persistent_variant(int bits, int bt, bool f32) {
+    if (f32) return bt == 256 ? kvar<uint32_t, 256, true>() : kvar<uint32_t, 512, true>();
     if (bits == 32) {
         if (bt == 128) return kvar<uint32_t, 128>();
         if (bt == 512) return kvar<uint32_t, 512>();
@@ -292,6 +294,15 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
 }
 
 unsigned heuristic_k(const sssp_graph* g) {
+    if (g->f32) {  // Delta = 2^(k - kFloatBias): ring span max_w / B in float
+        union {
+            unsigned u;
+            float f;
+        } mw{g->max_w};
+        const double q = (double)mw.f / (double)g->opts.num_buckets;
+        const long e = q > 0 ? std::lround(std::log2(q)) : -40;
+        return (unsigned)std::min<long>(std::max<long>(e + kFloatBias, 0), 190);
+    }
     switch (g->opts.delta_heuristic) {
         case SSSP_DELTA_H_NEARFAR: return g->heur_k_nf;
         case SSSP_DELTA_H_MAXW_OVER_D: return g->heur_k_md;
@@ -303,11 +314,12 @@ unsigned heuristic_k(const sssp_graph* g) {
 // `conc` workspaces share the GPU: each persistent grid gets 1/conc of the CTAs.
 // (The kernel never waits on a CTA that has not started -- no grid barrier --
 // so co-residency is not required; one slot launches cooperatively anyway.)
-template <typename DistT>
-sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, unsigned long long* out_dev, cudaStream_t s,
-                       int bits, unsigned k0, unsigned conc) {
-    const unsigned bt = g->opts.block_threads ? g->opts.block_threads : 512;
-    const KVariant kv = persistent_variant(bits, (int)bt);
+template <typename DistT, bool kF>
+sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_dev, cudaStream_t s, int bits,
+                       unsigned k0, unsigned conc) {
+    unsigned bt = g->opts.block_threads ? g->opts.block_threads : 512;
+    if (kF && bt != 256) bt = 512;  // float variants are built for 256/512-thread CTAs
+    const KVariant kv = persistent_variant(bits, (int)bt, kF);
     void* fn = kv.fn;
     CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kv.smem), "smem attribute");
     int occ = 0;
@@ -316,7 +328,7 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, unsigned lo
     unsigned grid = (unsigned)(occ * g->sm_count);
     if (g->opts.grid_ctas && g->opts.grid_ctas < grid) grid = g->opts.grid_ctas;
     grid = std::max(1u, grid / conc);
-    const unsigned k_max = bits == 32 ? 31u : 63u;
+    const unsigned k_max = kF ? 190u : (bits == 32 ? 31u : 63u);
     unsigned k = std::min(k0, k_max);
     const unsigned A0 = g->opts.active_init ? g->opts.active_init : 1u;
     Head h0{0ull, pack_meta(0, k, A0, 0, 0)};
@@ -335,7 +347,10 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, unsigned lo
         CK(cudaLaunchKernel(fn, dim3(grid), dim3(bt), args, kv.smem, s), "persistent kernel launch");
     }
     CK(cudaEventRecord(w.ev[2], s), "event");
-    finalize_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, out_dev, g->n, g->d_off, p.ctl);
+    if constexpr (kF)
+        finalize_f32_kernel<<<aux_grid, 256, 0, s>>>((const unsigned*)p.dist, (float*)out_dev, g->n, g->d_off, p.ctl);
+    else
+        finalize_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, (unsigned long long*)out_dev, g->n, g->d_off, p.ctl);
     CK(cudaGetLastError(), "finalize kernel launch");
     CK(cudaEventRecord(w.ev[3], s), "event");
     CK(cudaMemcpyAsync(w.h_ctl, w.ctl.p, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "status copy");
@@ -358,8 +373,9 @@ sssp_status ensure_nf(sssp_graph* g, Workspace& w, int item_bytes, unsigned long
 }
 
 template <typename DistT>
-sssp_status launch_nf(sssp_graph* g, Workspace& w, uint32_t source, unsigned long long* out_dev, cudaStream_t s,
+sssp_status launch_nf(sssp_graph* g, Workspace& w, uint32_t source, void* out_dev_v, cudaStream_t s,
                       int bits, unsigned k0) {
+    unsigned long long* out_dev = (unsigned long long*)out_dev_v;
     const int ib = bits == 32 ? 8 : 16;
     sssp_status st = ensure_nf(g, w, ib, w.nf_cap ? w.nf_cap : 2 * default_cap(g));
     if (st) return st;
@@ -401,8 +417,17 @@ sssp_status launch_nf(sssp_graph* g, Workspace& w, uint32_t source, unsigned lon
     return SSSP_OK;
 }
 
-sssp_status launch_attempt(sssp_graph* g, Workspace& w, uint32_t source, unsigned long long* out_dev, cudaStream_t s,
+sssp_status launch_attempt(sssp_graph* g, Workspace& w, uint32_t source, void* out_dev, cudaStream_t s,
                            int bits, unsigned conc) {
+    if (g->f32) {
+        if (g->opts.algorithm == SSSP_ALGO_NEAR_FAR)
+            return fail(SSSP_ERR_INVALID_ARGUMENT, "the Near-Far ablation supports integer weights only");
+        const unsigned k0 = g->opts.delta_init ? kFloatBias + ilog2_round((double)g->opts.delta_init) : heuristic_k(g);
+        sssp_status st = ensure_ring(g, w, 8, w.cap ? w.cap : default_cap(g));
+        if (st) return st;
+        if ((st = ensure_trace(g, w))) return st;
+        return launch_one<uint32_t, true>(g, w, source, out_dev, s, 32, k0, conc);
+    }
     if (g->opts.algorithm == SSSP_ALGO_NEAR_FAR) {
         // static Delta: the Near-Far rule unless given
         const unsigned k0 = g->opts.delta_init ? ilog2_round((double)g->opts.delta_init) : g->heur_k_nf;
@@ -413,8 +438,8 @@ sssp_status launch_attempt(sssp_graph* g, Workspace& w, uint32_t source, unsigne
     sssp_status st = ensure_ring(g, w, bits == 32 ? 8 : 16, w.cap ? w.cap : default_cap(g));
     if (st) return st;
     if ((st = ensure_trace(g, w))) return st;
-    if (bits == 32) return launch_one<uint32_t>(g, w, source, out_dev, s, 32, k0, conc);
-    return launch_one<unsigned long long>(g, w, source, out_dev, s, 64, k0, conc);
+    if (bits == 32) return launch_one<uint32_t, false>(g, w, source, out_dev, s, 32, k0, conc);
+    return launch_one<unsigned long long, false>(g, w, source, out_dev, s, 64, k0, conc);
 }
 
 void accumulate(sssp_graph* g, Workspace& w, const Ctl& c, int bits) {
@@ -485,7 +510,7 @@ sssp_status settle_attempt(sssp_graph* g, Workspace& w, cudaStream_t s, int& bit
 }
 
 // Synchronous run of one source on one workspace, with retry.
-sssp_status run_one_sync(sssp_graph* g, Workspace& w, uint32_t source, unsigned long long* out_dev, cudaStream_t s,
+sssp_status run_one_sync(sssp_graph* g, Workspace& w, uint32_t source, void* out_dev, cudaStream_t s,
                          unsigned conc) {
     int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
     for (int attempt = 0; attempt < 24; ++attempt) {
@@ -518,7 +543,7 @@ sssp_status classify_out(sssp_graph* g, const void* ptr, bool* is_dev) {
 
 // Concurrent batch (device dist_out): groups of c sources, one per workspace
 // and stream; every attempt of a group is launched before any is awaited.
-sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, unsigned long long* out,
+sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, char* out, size_t esz,
                            cudaStream_t caller, unsigned c) {
     sssp_status st = ensure_slots(g, c);
     if (st) return st;
@@ -529,7 +554,8 @@ sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, u
         const unsigned cnt = std::min<uint32_t>(c, k - i0);
         int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
         for (unsigned j = 0; j < cnt && st == SSSP_OK; ++j)
-            st = launch_attempt(g, *g->ws[j], sources[i0 + j], out + (size_t)(i0 + j) * g->n, slot_stream(j), bits, c);
+            st = launch_attempt(g, *g->ws[j], sources[i0 + j], out + (size_t)(i0 + j) * g->n * esz, slot_stream(j),
+                                bits, c);
         for (unsigned j = 0; j < cnt && st == SSSP_OK; ++j) {
             const cudaError_t e = cudaStreamSynchronize(slot_stream(j));
             if (e != cudaSuccess) {
@@ -540,7 +566,8 @@ sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, u
             bool done = false;
             st = settle_attempt(g, *g->ws[j], slot_stream(j), b, 0, &done);
             if (st == SSSP_OK && !done)  // recoverable: redo this source alone (still concurrent-sized grid)
-                st = run_one_sync(g, *g->ws[j], sources[i0 + j], out + (size_t)(i0 + j) * g->n, slot_stream(j), c);
+                st = run_one_sync(g, *g->ws[j], sources[i0 + j], out + (size_t)(i0 + j) * g->n * esz, slot_stream(j),
+                                  c);
         }
     }
     for (unsigned j = 1; j < c; ++j) {
@@ -550,8 +577,13 @@ sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, u
     return st;
 }
 
-sssp_status run_many(sssp_graph* g, const uint32_t* sources, uint32_t k, uint64_t* dist_out, sssp_stream_t stream) {
+sssp_status run_many(sssp_graph* g, const uint32_t* sources, uint32_t k, void* dist_out, bool f32_out,
+                     sssp_stream_t stream) {
     if (!g || !dist_out || (k && !sources)) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL argument");
+    if (f32_out != g->f32)
+        return fail(SSSP_ERR_INVALID_ARGUMENT, g->f32 ? "float32-weight graph: use sssp_run_f32 / sssp_run_batch_f32"
+                                                      : "integer-weight graph: use sssp_run / sssp_run_batch");
+    const size_t esz = g->f32 ? 4 : 8;
     if (k == 0) return fail(SSSP_ERR_INVALID_ARGUMENT, "k == 0");
     for (uint32_t i = 0; i < k; ++i)
         if (sources[i] >= g->n) return fail(SSSP_ERR_INVALID_ARGUMENT, "source " + std::to_string(sources[i]) + " >= n");
@@ -579,11 +611,10 @@ sssp_status run_many(sssp_graph* g, const uint32_t* sources, uint32_t k, uint64_
     }
     cudaEventRecord(g->bev[0], s);
     if (is_dev && c > 1) {
-        st = run_concurrent(g, sources, k, (unsigned long long*)dist_out, s, c);
+        st = run_concurrent(g, sources, k, (char*)dist_out, esz, s, c);
     } else {
         for (uint32_t i = 0; i < k && st == SSSP_OK; ++i) {
-            unsigned long long* out = is_dev ? (unsigned long long*)dist_out + (size_t)i * g->n
-                                             : (unsigned long long*)g->hostout.p;
+            void* out = is_dev ? (void*)((char*)dist_out + (size_t)i * g->n * esz) : g->hostout.p;
             if (async) {
                 const int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
                 st = launch_attempt(g, w0, sources[i], out, s, bits, 1);
@@ -594,8 +625,8 @@ sssp_status run_many(sssp_graph* g, const uint32_t* sources, uint32_t k, uint64_
             } else {
                 st = run_one_sync(g, w0, sources[i], out, s, 1);
                 if (st == SSSP_OK && !is_dev) {
-                    cudaError_t e = cudaMemcpyAsync((unsigned long long*)dist_out + (size_t)i * g->n, out,
-                                                    (size_t)g->n * 8, cudaMemcpyDeviceToHost, s);
+                    cudaError_t e = cudaMemcpyAsync((char*)dist_out + (size_t)i * g->n * esz, out, (size_t)g->n * esz,
+                                                    cudaMemcpyDeviceToHost, s);
                     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
                     if (e != cudaSuccess) st = cuda_fail(e, "copying dist to host");
                 }
@@ -647,8 +678,11 @@ void sssp_options_default(sssp_options* o) {
     o->concurrent_sources = 1;
 }
 
-sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offsets, const uint32_t* col,
-                              const uint32_t* w, const sssp_options* opts, sssp_graph** out) {
+}  // extern "C"
+
+namespace {
+sssp_status create_impl(uint32_t n, uint64_t m, const uint64_t* row_offsets, const uint32_t* col, const uint32_t* w,
+                        bool f32, const sssp_options* opts, sssp_graph** out) {
     if (!out) return fail(SSSP_ERR_INVALID_ARGUMENT, "out is NULL");
     *out = nullptr;
     if (!row_offsets || (m && (!col || !w))) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL CSR array");
@@ -675,6 +709,7 @@ sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offset
     g->m = m;
     g->opts = o;
     g->sm_count = prop.multiProcessorCount;
+    g->f32 = f32;
     g->persist_max = prop.persistingL2CacheMaxSize > 0 ? (size_t)prop.persistingL2CacheMaxSize : 0;
     auto bail = [&](sssp_status s2) {
         sssp_graph_destroy(g);
@@ -697,7 +732,7 @@ sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offset
     CKG(cudaMalloc(&g->d_adj, std::max<size_t>(m, 1) * sizeof(uint2)), "allocating arcs");
     CKG(cudaMalloc(&g->scratch.p, 64), "scratch");
     unsigned long long* d_bad = (unsigned long long*)g->scratch.p;  // [0],[1] bad idx, [2] sum_w, [3] max_w
-    unsigned long long init_scr[4] = {~0ull, ~0ull, 0, 0};
+    unsigned long long init_scr[5] = {~0ull, ~0ull, 0, 0, ~0ull};  // [4] first bad float weight
     CKG(cudaMemcpy(d_bad, init_scr, sizeof(init_scr), cudaMemcpyHostToDevice), "scratch init");
     const unsigned aux_grid = (unsigned)g->sm_count * 8;
     if (m) {
@@ -712,7 +747,10 @@ sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offset
         if (e == cudaSuccess) e = cudaMemcpy(d_w, w, m * 4, cudaMemcpyDefault);
         if (e == cudaSuccess) {
             validate_csr_kernel<<<aux_grid, 256>>>(g->d_off, d_col, n, m, d_bad);
-            interleave_kernel<<<aux_grid, 256>>>(d_col, d_w, g->d_adj, m, d_bad + 2, (unsigned*)(d_bad + 3));
+            if (f32)
+                interleave_f32_kernel<<<aux_grid, 256>>>(d_col, d_w, g->d_adj, m, d_bad + 4, (unsigned*)(d_bad + 3));
+            else
+                interleave_kernel<<<aux_grid, 256>>>(d_col, d_w, g->d_adj, m, d_bad + 2, (unsigned*)(d_bad + 3));
             e = cudaDeviceSynchronize();
         }
         cudaFree(d_col);
@@ -722,17 +760,19 @@ sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offset
         validate_csr_kernel<<<aux_grid, 256>>>(g->d_off, nullptr, n, 0, d_bad);
         CKG(cudaDeviceSynchronize(), "validating the CSR");
     }
-    unsigned long long scr[4];
+    unsigned long long scr[5];
     CKG(cudaMemcpy(scr, d_bad, sizeof(scr), cudaMemcpyDeviceToHost), "reading validation result");
     if (scr[0] != ~0ull)
         return bail(fail(SSSP_ERR_INVALID_GRAPH, "row_offsets decreasing at index " + std::to_string(scr[0])));
     if (scr[1] != ~0ull)
         return bail(fail(SSSP_ERR_INVALID_GRAPH, "col[" + std::to_string(scr[1]) + "] >= n"));
+    if (scr[4] != ~0ull)
+        return bail(fail(SSSP_ERR_INVALID_GRAPH, "w[" + std::to_string(scr[4]) + "] is negative or NaN"));
     g->sum_w = scr[2];
     g->max_w = (uint32_t)scr[3];
     // initial Delta (reading R3): max_w / D (Meyer-Sanders' Theta(1/d) rule for Delta-stepping [15]),
     // or the Near-Far rule C * W / D with W = average weight, D = average degree, C = 32
-    if (m && g->sum_w) {
+    if (m && g->sum_w && !f32) {
         const double W = (double)g->sum_w / (double)m, D = (double)m / (double)n;
         g->heur_k_nf = std::min(ilog2_round(32.0 * W / D), 63u);
         g->heur_k_md = std::min(ilog2_round((double)g->max_w / std::max(D, 1.0)), 63u);
@@ -748,6 +788,19 @@ sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offset
 #undef CKG
     *out = g;
     return SSSP_OK;
+}
+}  // namespace
+
+extern "C" {
+
+sssp_status sssp_graph_create(uint32_t n, uint64_t m, const uint64_t* row_offsets, const uint32_t* col,
+                              const uint32_t* w, const sssp_options* opts, sssp_graph** out) {
+    return create_impl(n, m, row_offsets, col, w, false, opts, out);
+}
+
+sssp_status sssp_graph_create_f32(uint32_t n, uint64_t m, const uint64_t* row_offsets, const uint32_t* col,
+                                  const float* w, const sssp_options* opts, sssp_graph** out) {
+    return create_impl(n, m, row_offsets, col, (const uint32_t*)w, true, opts, out);
 }
 
 sssp_status sssp_graph_destroy(sssp_graph* g) {
@@ -790,12 +843,21 @@ sssp_status sssp_set_options(sssp_graph* g, const sssp_options* opts) {
 }
 
 sssp_status sssp_run(sssp_graph* g, uint32_t source, uint64_t* dist_out, sssp_stream_t stream) {
-    return run_many(g, &source, 1, dist_out, stream);
+    return run_many(g, &source, 1, dist_out, false, stream);
 }
 
 sssp_status sssp_run_batch(sssp_graph* g, const uint32_t* sources, uint32_t k, uint64_t* dist_out,
                            sssp_stream_t stream) {
-    return run_many(g, sources, k, dist_out, stream);
+    return run_many(g, sources, k, dist_out, false, stream);
+}
+
+sssp_status sssp_run_f32(sssp_graph* g, uint32_t source, float* dist_out, sssp_stream_t stream) {
+    return run_many(g, &source, 1, dist_out, true, stream);
+}
+
+sssp_status sssp_run_batch_f32(sssp_graph* g, const uint32_t* sources, uint32_t k, float* dist_out,
+                               sssp_stream_t stream) {
+    return run_many(g, sources, k, dist_out, true, stream);
 }
 
 sssp_status sssp_get_stats(sssp_graph* g, sssp_stats* out) {

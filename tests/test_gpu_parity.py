@@ -299,3 +299,61 @@ def test_near_far_u64_and_golden():
         gg2 = gg.from_arcs(fx["n"], fx["arcs"])
         d, _ = gpu_dist(gg2, fx["source"], algorithm=sssp.SSSP_ALGO_NEAR_FAR)
         assert [int(x) for x in d] == fx["dist"]
+
+
+# ----------------------------------------------------------------- NEXT-3: float32 weights
+def check_f32(g, wf, s, **opt):
+    ref, V, E = oracle.dijkstra_f32(g, wf, int(s))
+    G = sssp.Graph.from_csr(g, weights=wf, **opt)
+    d = G.run(int(s)).cpu().numpy()
+    st = G.stats()
+    G.close()
+    bad = np.flatnonzero(d.view(np.uint32) != ref.view(np.uint32))
+    assert bad.size == 0, f"{bad.size} mismatches, first {bad[:5]} gpu={d[bad[:5]]} ref={ref[bad[:5]]} {opt}"
+    assert st["reachable"] == V and st["reach_edges"] == E
+    return st
+
+
+@pytest.mark.parametrize("config,lo,hi", [("road", 0.0, 1.0), ("rmat", 1.0, 255.0), ("er", 0.0, 1e-3),
+                                          ("road", 100.0, 1e6)])
+def test_float_weights_scaled(config, lo, hi):
+    g = gg.make(config, scale_down=8)
+    wf = gg.float_weights(g, lo, hi, seed=11)
+    for s in gg.config_sources(config, g, 2):
+        check_f32(g, wf, s)
+
+
+@pytest.mark.parametrize("opt", [dict(delta_mode=1, delta_init=1), dict(delta_mode=1, delta_init=1 << 20),
+                                 dict(ring_items=64), dict(grid_ctas=3), dict(block_threads=256),
+                                 dict(flags=sssp.SSSP_FLAG_NO_LOCAL), dict(concurrent_sources=2)],
+                         ids=lambda o: ",".join(f"{k}={v}" for k, v in o.items()))
+def test_float_weights_perturbed(opt):
+    g = gg.make("rmat", scale_down=10)
+    wf = gg.float_weights(g, 0.0, 1.0, seed=3)
+    check_f32(g, wf, int(gg.config_sources("rmat", g, 1)[0]), **opt)
+
+
+def test_float_weights_full_size_road():
+    g = gg.make("road")
+    wf = gg.float_weights(g, 0.0, 1.0, seed=2)
+    st = check_f32(g, wf, int(gg.config_sources("road", g, 1)[0]))
+    assert st["edges_relaxed"] <= 3 * st["reach_edges"]
+
+
+def test_float_rounding_fixture_and_errors():
+    F32 = np.float32
+    one_ulp = np.nextafter(F32(1.0), F32(2.0))
+    g = gg.from_arcs(3, [(0, 1, 0), (0, 2, 0), (1, 2, 0)])   # CSR order: (0,1) (0,2) (1,2)
+    wf = np.array([1.0, one_ulp, 2.0 ** -24], dtype=F32)
+    G = sssp.Graph.from_csr(g, weights=wf)
+    d = G.run(0).cpu().numpy()
+    assert d.tolist() == [0.0, 1.0, 1.0]                       # 1 + 2^-24 rounds to 1.0
+    with pytest.raises(sssp.SSSPError) as e:
+        sssp.Graph.from_csr(g, weights=np.array([1.0, -2.0, 0.5], dtype=F32))
+    assert e.value.status == 2 and "w[1]" in e.value.detail
+    with pytest.raises(sssp.SSSPError) as e:
+        sssp.lib().sssp_run(G._h, 0, torch.empty(3, dtype=torch.int64, device="cuda").data_ptr(), 0)
+        sssp._check(sssp.lib().sssp_run(G._h, 0, torch.empty(3, dtype=torch.int64, device="cuda").data_ptr(), 0))
+    assert e.value.status == 1
+    nz = sssp.Graph.from_csr(g, weights=np.array([-0.0, 1.0, 1.0], dtype=F32))   # -0.0 folds to +0.0
+    assert nz.run(0).cpu().numpy().tolist() == [0.0, 0.0, 1.0]
