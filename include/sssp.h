@@ -129,7 +129,7 @@ typedef struct sssp_options {
     uint32_t max_backoff_ns;   /* idle CTAs back off exponentially up to this (0 = auto = 2048) */
     uint32_t startup_permille; /* the controller may not grow Delta before this share of the vertices
                                   has been expanded or 32 head switches have happened (start-up
-                                  frontiers are always small); default 2 */
+                                  frontiers are always small); default 20 (2%) */
     uint32_t concurrent_sources; /* sssp_run_batch: sources in flight at once on this GPU (NEXT-1), each
                                   with its own workspace (dist, bucket ring, counters) and stream and
                                   1/c of the SMs; the CSR is shared.  0/1 = one at a time */

@@ -121,10 +121,13 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
     const bool high = util * 100ull > (unsigned long long)p.util_hi_pct * T;
     const bool beyond = (total - win) > win;  // more work waits outside the active window
     // waste: recent re-expansions high AND the run as a whole already above 2x
-    const bool wasteful = waste_known && waste > p.waste_hi && ratio_x100 > 200;
+    // (both need the start-up gate: early samples are tiny and noisy)
+    const bool wasteful = progressed && waste_known && waste > p.waste_hi && ratio_x100 > 200;
     // frugal: recent and cumulative re-expansion both low
     // (no growth during the start-up transient: the first frontier is always small)
-    const bool frugal = waste_known && waste < p.waste_lo && ratio_x100 < 125 && progressed;
+    // (an unmeasurable waste -- too few expansions in the window -- means the run
+    // is crawling: growth is allowed once the start-up gate is open)
+    const bool frugal = (!waste_known || waste < p.waste_lo) && ratio_x100 < 150 && progressed;
     const bool clipping = (total >= 64 && tail * 100 >= (long long)p.clip_pct * total) || (clip_known && clip >= 500);
     d.flags = (low ? 1u : 0u) | (high ? 2u : 0u) | (beyond ? 4u : 0u) | (wasteful ? 8u : 0u) |
               (frugal ? 16u : 0u) | (clipping ? 32u : 0u) | (waste_known ? 64u : 0u) | (progressed ? 128u : 0u) |
@@ -141,7 +144,8 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
             d.k = k + 1;
             d.changed = true;
         }
-    } else if (d.since * 4 >= p.settle && low && frugal && beyond && waste * 8 < p.waste_lo && k < p.k_max) {
+    } else if (d.since * 4 >= p.settle && low && frugal && beyond && (!waste_known || waste * 8 < p.waste_lo) &&
+               k < p.k_max) {
         d.k = k + 1;  // essentially no re-expansion yet: grow with a quarter of the settling time
         d.changed = true;
     }

@@ -665,7 +665,7 @@ void sssp_options_default(sssp_options* o) {
     o->waste_lo_permille = 450;    // reading R6: grow Delta only while < 45% of expansions are repeats
     o->waste_hi_permille = 500;    //             shrink it while > 50% are (work <~ 2x Dijkstra)
     o->period_us = 20;
-    o->startup_permille = 2;
+    o->startup_permille = 20;
     o->dist_bits = 0;
     o->ring_items = 0;
     o->flags = 0;
