@@ -365,7 +365,6 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
     using Raw = typename IT::Raw;
     using L = Smem<DistT, BT, EPT, W>;
     constexpr int kStage = L::kStage;
-    constexpr int kRound = BT * EPT;  // arcs per CTA round
     constexpr int kWarps = BT / 32;
     constexpr int kPer = W / BT;      // window positions per thread in the owner scan
     constexpr unsigned long long kInf = (unsigned long long)DistInf<DistT>::value;
@@ -386,7 +385,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
     __shared__ unsigned s_cnt[kMaxBuckets];
     __shared__ unsigned long long s_base[kMaxBuckets];
     __shared__ unsigned s_wsum[kWarps];
-    __shared__ unsigned s_total, s_E, s_got, s_slot, s_lnext;
+    __shared__ unsigned s_total, s_E, s_got, s_slot, s_lnext, s_direct;
     __shared__ int s_cmd;
     __shared__ unsigned long long s_idx;
     __shared__ Head s_head;
@@ -406,6 +405,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
     if (tid == 0) {
         s_total = 0;
         s_lnext = 0;
+        s_direct = 0;
     }
     const bool prof = p.prof != 0 && tid == 0;
     const unsigned long long pol_stream = policy_evict_first();  // arcs, row offsets
@@ -587,147 +587,71 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
             tw = 0;
         }
 
-        // latency fast path (road-like graphs): a batch whose arcs fit one round
-        // skips the owner map + async window and the L2 filter load -- two
-        // dependent steps fewer per hop; arcs are loaded directly, relaxed by atomicMin
-        const bool small = E <= (unsigned)kRound;
-        if (small) __syncthreads();  // publishes s_scan
-        for (unsigned wbase = 0; wbase < E; wbase += W) {
-            const unsigned Ew = (E - wbase) < (unsigned)W ? (E - wbase) : (unsigned)W;
-            const long long tw0 = prof ? clock64() : 0;
-            if (!small) {
-            // ------------------------------------------------ owner of every window position
-            // zero, mark row starts, inclusive prefix-max (rows are in scan order)
-            {
-                unsigned short* ow = s_owner + tid * kPer;
-#pragma unroll
-                for (int i = 0; i < kPer; ++i) ow[i] = 0;
-            }
-            __syncthreads();  // (also publishes s_scan)
-            if (tid < (int)got && deg) {
-                const unsigned st = s_scan[tid];
-                if (st > wbase && st < wbase + Ew) s_owner[st - wbase] = (unsigned short)tid;
-            }
-            if (tid == 0) {  // owner of the window's first arc: largest i with scan[i] <= wbase
-                unsigned lo = 0, hi = got - 1;
-                while (lo < hi) {
-                    const unsigned mid = (lo + hi + 1) >> 1;
-                    if (s_scan[mid] <= wbase) lo = mid;
-                    else hi = mid - 1;
-                }
-                s_owner[0] = (unsigned short)lo;
-            }
-            __syncthreads();
-            {
-                unsigned short* ow = s_owner + tid * kPer;
-                unsigned run[kPer];
-                unsigned m = 0;
-#pragma unroll
-                for (int i = 0; i < kPer; ++i) {
-                    m = ow[i] > m ? ow[i] : m;
-                    run[i] = m;
-                }
-                unsigned inc = m;  // warp inclusive max-scan of per-thread maxima
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const unsigned y = __shfl_up_sync(FULL, inc, o);
-                    if (lane >= o) inc = y > inc ? y : inc;
-                }
-                unsigned excl = __shfl_up_sync(FULL, inc, 1);
-                if (lane == 0) excl = 0;
-                if (lane == 31) s_wsum[warp] = inc;
-                __syncthreads();
-                unsigned wpre = 0;
-#pragma unroll
-                for (int w2 = 0; w2 < kWarps; ++w2)
-                    if (w2 < warp) wpre = s_wsum[w2] > wpre ? s_wsum[w2] : wpre;
-                const unsigned carry = excl > wpre ? excl : wpre;
-#pragma unroll
-                for (int i = 0; i < kPer; ++i) ow[i] = (unsigned short)(run[i] > carry ? run[i] : carry);
-            }
-            __syncthreads();
-            // ------------------------------------------------ async arc prefetch: the
-            // whole window in flight at once (LDGSTS), coalesced along each row
-            for (unsigned q = tid; q < Ew; q += BT) {
-                const unsigned o = s_owner[q];
-                cp_async_8(s_arc_addr + q * 8u, p.adj + s_ebeg[o] + (wbase + q - s_scan[o]), pol_stream);
-            }
-            cp_async_wait_all();
-            __syncthreads();
-            if (prof) {
-                tw += clock64() - tw0;
-                s_prof[PR_N_WINDOW] += 1;
-            }
-            }  // !small
-
-            // ------------------------------------------------ relax + push (rounds)
-            for (unsigned rbase = 0; rbase < Ew; rbase += kRound) {
+        __syncthreads();  // publishes s_scan / s_d / s_ebeg
+        // ---------------------------------------------------- stream the batch's arcs
+        // Warp w owns a contiguous slice of the batch's arc space and streams through
+        // it with no CTA barrier (warps drift and keep the L1TEX queue busy); lanes
+        // take consecutive arcs (coalesced along rows), EPT in flight per lane; the
+        // owner of an arc is found by binary search over the CTA scan in shared memory.
+        // Tiny batches (latency regime, road-like graphs) skip the L2 filter load.
+        {
+            const bool tiny = E <= (unsigned)BT;
+            const unsigned per = (E + kWarps - 1) / kWarps;
+            const unsigned slice = (per + 31) / 32 * 32;  // small batches spread over many warps
+            const unsigned wb = warp * slice;
+            const unsigned we = (wb + slice) < E ? (wb + slice) : E;
+            for (unsigned base = wb; base < we; base += 32 * EPT) {
+                unsigned own[EPT];
                 uint2 a[EPT];
                 unsigned long long nd[EPT];
                 bool push[EPT];
                 DistT cur[EPT];
-                if (small) {
-                    unsigned own[EPT];
 #pragma unroll
-                    for (int j = 0; j < EPT; ++j) {  // owner = largest i with scan[i] <= q
-                        const unsigned q = j * BT + tid;
-                        unsigned lo = 0, hi = got - 1;
-                        if (q < Ew) {
-                            while (lo < hi) {
-                                const unsigned mid = (lo + hi + 1) >> 1;
-                                if (s_scan[mid] <= q) lo = mid;
-                                else hi = mid - 1;
-                            }
-                        }
-                        own[j] = lo;
-                    }
-#pragma unroll
-                    for (int j = 0; j < EPT; ++j) {  // EPT independent arc loads in flight
-                        const unsigned q = j * BT + tid;
-                        if (q < Ew) {
-                            a[j] = ld_stream_u2(p.adj + s_ebeg[own[j]] + (q - s_scan[own[j]]), pol_stream);
-                            nd[j] = relax_sum<kF>((unsigned long long)s_d[own[j]], a[j].y);
-                            cur[j] = DistInf<DistT>::value;  // tiny batch: straight to atomicMin
-                        } else {
-                            a[j] = make_uint2(0u, 0u);
-                            nd[j] = kInf;
-                            cur[j] = (DistT)0;
+                for (int j = 0; j < EPT; ++j) {  // owner = largest i with scan[i] <= e
+                    const unsigned e = base + j * 32 + lane;
+                    unsigned lo = 0, hi = got - 1;
+                    if (e < we) {
+                        while (lo < hi) {
+                            const unsigned mid = (lo + hi + 1) >> 1;
+                            if (s_scan[mid] <= e) lo = mid;
+                            else hi = mid - 1;
                         }
                     }
-                    if (E > (unsigned)BT) {  // more than one arc per thread: keep the L2 filter
-#pragma unroll
-                        for (int j = 0; j < EPT; ++j)
-                            if (nd[j] < kInf) cur[j] = ld_keep(p.dist + a[j].x, pol_keep);
-                    }
-                } else {
-#pragma unroll
-                    for (int j = 0; j < EPT; ++j) {
-                        const unsigned q = rbase + j * BT + tid;
-                        if (q < Ew) {
-                            a[j] = s_arc[q];
-                            nd[j] = relax_sum<kF>((unsigned long long)s_d[s_owner[q]], a[j].y);
-                        } else {
-                            a[j] = make_uint2(0u, 0u);
-                            nd[j] = kInf;
-                        }
-                    }
-#pragma unroll
-                    for (int j = 0; j < EPT; ++j)  // EPT independent L2 gathers in flight
-                        cur[j] = nd[j] < kInf ? ld_keep(p.dist + a[j].x, pol_keep) : (DistT)0;
+                    own[j] = lo;
                 }
 #pragma unroll
-                for (int j = 0; j < EPT; ++j) {
-                    const unsigned q = rbase + j * BT + tid;
-                    push[j] = false;
-                    if (q < Ew) {
+                for (int j = 0; j < EPT; ++j) {  // EPT independent arc loads in flight
+                    const unsigned e = base + j * 32 + lane;
+                    if (e < we) {
+                        a[j] = ld_stream_u2(p.adj + s_ebeg[own[j]] + (e - s_scan[own[j]]), pol_stream);
+                        nd[j] = relax_sum<kF>((unsigned long long)s_d[own[j]], a[j].y);
+                    } else {
+                        a[j] = make_uint2(0u, 0u);
+                        nd[j] = kInf;
+                    }
+                }
+#pragma unroll
+                for (int j = 0; j < EPT; ++j)  // EPT independent L2 gathers in flight
+                    cur[j] = (nd[j] < kInf && !tiny) ? ld_keep(p.dist + a[j].x, pol_keep)
+                                                     : (nd[j] < kInf ? DistInf<DistT>::value : (DistT)0);
+                DistT old[EPT];
+                bool tried[EPT];
+#pragma unroll
+                for (int j = 0; j < EPT; ++j) {  // all atomics issued before any result is used
+                    const unsigned e = base + j * 32 + lane;
+                    tried[j] = false;
+                    old[j] = (DistT)0;
+                    if (e < we) {
                         if (sum_unusable<kF>(nd[j], kInf)) {
                             if (!kF) atomicOr(&p.ctl->status, kStDistOverflow);  // 32-bit distances insufficient
                         } else if (nd[j] < (unsigned long long)cur[j]) {
-                            const DistT old = atomic_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
-                            push[j] = nd[j] < (unsigned long long)old;
+                            old[j] = atomic_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
+                            tried[j] = true;
                         }
                     }
                 }
+#pragma unroll
+                for (int j = 0; j < EPT; ++j) push[j] = tried[j] && nd[j] < (unsigned long long)old[j];
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {
                     if (!__any_sync(FULL, push[j])) continue;
@@ -750,83 +674,129 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                     }
                     const bool pg = push[j] && !kept;
                     const unsigned act = __ballot_sync(FULL, pg);
-                    if (pg) {  // warp-aggregated staging for the ring
-                        const int leader = __ffs(act) - 1;
-                        unsigned pos = 0;
-                        if (lane == leader) pos = atomicAdd(&s_total, (unsigned)__popc(act));
-                        pos = __shfl_sync(act, pos, leader) + __popc(act & lt_mask);
-                        const unsigned peers = __match_any_sync(act, o);
-                        const int pl = __ffs(peers) - 1;
-                        unsigned r0 = 0;
-                        if (lane == pl) r0 = atomicAdd(&s_cnt[o], (unsigned)__popc(peers));
-                        r0 = __shfl_sync(peers, r0, pl) + __popc(peers & lt_mask);
-                        s_items[pos] = IT::make(a[j].x, nd[j]);
-                        s_soff[pos] = (unsigned char)o;
-                        s_rank[pos] = (unsigned short)r0;
-                    }
-                }
-                __syncthreads();
-                const unsigned total = s_total;
-                if (prof) s_prof[PR_N_ROUND] += 1;
-                const bool last = (wbase + rbase + kRound >= E);
-                if (total > (unsigned)(kStage - kRound) || (last && total > 0)) {
-                    // ------------------------------------------------ flush to the ring
-                    const long long tf = prof ? clock64() : 0;
-                    if (warp == 0 && lane < (int)p.nb) {
-                        const unsigned c = s_cnt[lane];
-                        if (p.dynamic) {
-                            if (lane == 0) atomicAdd(&p.ctl->g_push, (unsigned long long)total);
-                            if (lane == (int)nbm && c) atomicAdd(&p.ctl->g_clip, (unsigned long long)c);
+                    if (!act) continue;
+                    // warp-aggregated staging slot for the CTA flush at batch end
+                    const int leader = __ffs(act) - 1;
+                    const unsigned nact = (unsigned)__popc(act);
+                    unsigned pos = 0;
+                    if (lane == leader) pos = atomicAdd(&s_total, nact);
+                    pos = __shfl_sync(FULL, pos, leader);
+                    if (pos + nact <= (unsigned)kStage) {
+                        if (pg) {
+                            const unsigned peers = __match_any_sync(act, o);
+                            const int pl = __ffs(peers) - 1;
+                            unsigned r0 = 0;
+                            if (lane == pl) r0 = atomicAdd(&s_cnt[o], (unsigned)__popc(peers));
+                            r0 = __shfl_sync(peers, r0, pl) + __popc(peers & lt_mask);
+                            const unsigned my = pos + __popc(act & lt_mask);
+                            s_items[my] = IT::make(a[j].x, nd[j]);
+                            s_soff[my] = (unsigned char)o;
+                            s_rank[my] = (unsigned short)r0;
                         }
-                        if (c) {
-                            const unsigned sl = (hs + lane) & nbm;
-                            // returning atomic: the reserve (which also counts the children for
-                            // termination) is performed before this CTA's completion atomic
-                            const unsigned long long b = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
-                            s_base[lane] = b;
-                            if (b + c > p.cap) {  // lapping: previous occupants must be claimed
-                                const unsigned long long cl = ld_relaxed_u64(&p.bk[sl].claim.v);
-                                if (b + c - p.cap > cl) atomicOr(&p.ctl->status, kStRingOverflow);
+                    } else {
+                        // staging full (hubs): mark the slots this warp took as holes and
+                        // publish directly -- one reserve/avail pair per (warp, bucket)
+                        if (pg) {
+                            const unsigned my = pos + __popc(act & lt_mask);
+                            if (my < (unsigned)kStage) s_soff[my] = 0xFF;
+                            const unsigned peers = __match_any_sync(act, o);
+                            const int pl = __ffs(peers) - 1;
+                            const unsigned sl = (hs + o) & nbm;
+                            unsigned long long b0 = 0;
+                            if (lane == pl) {
+                                const unsigned c = (unsigned)__popc(peers);
+                                b0 = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
+                                if (b0 + c > p.cap) {
+                                    const unsigned long long cl = ld_relaxed_u64(&p.bk[sl].claim.v);
+                                    if (b0 + c - p.cap > cl) atomicOr(&p.ctl->status, kStRingOverflow);
+                                }
+                                atomicAdd(&s_direct, c);
                             }
-                        }
-                    }
-                    __syncthreads();
-                    for (unsigned i = tid; i < total; i += BT) {
-                        const unsigned o = s_soff[i];
-                        const unsigned sl = (hs + o) & nbm;
-                        const unsigned long long idx = s_base[o] + s_rank[i];
-                        char* sp = p.ring + ((size_t)sl * p.cap + (idx & (p.cap - 1))) * IT::kBytes;
-                        bool ok = true;
-                        if (idx >= p.cap) {  // wait for the previous lap's reader to clear it
-                            unsigned spins = 0;
-                            while (!IT::empty(sp)) {
-                                if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) {
-                                    ok = false;
-                                    break;
+                            b0 = __shfl_sync(peers, b0, pl);
+                            const unsigned long long idx = b0 + __popc(peers & lt_mask);
+                            char* sp = p.ring + ((size_t)sl * p.cap + (idx & (p.cap - 1))) * IT::kBytes;
+                            bool ok = true;
+                            if (idx >= p.cap) {
+                                unsigned spins = 0;
+                                while (!IT::empty(sp)) {
+                                    if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) {
+                                        ok = false;
+                                        break;
+                                    }
                                 }
                             }
+                            if (ok) IT::store(sp, IT::make(a[j].x, nd[j]));
+                            __syncwarp(peers);
+                            if (lane == pl) atomicAdd(&p.bk[sl].avail.v, (unsigned long long)__popc(peers));
                         }
-                        if (ok) IT::store(sp, s_items[i]);
-                    }
-                    __syncthreads();
-                    if (warp == 0 && lane < (int)p.nb) {
-                        const unsigned c = s_cnt[lane];
-                        if (c) {
-                            atomicAdd(&p.bk[(hs + lane) & nbm].avail.v, (unsigned long long)c);  // publish
-                            s_cnt[lane] = 0;
-                        }
-                    }
-                    if (tid == 0) {
-                        s_total = 0;
-                        c_push += total;
-                    }
-                    __syncthreads();
-                    if (prof) {
-                        tq += clock64() - tf;
-                        s_prof[PR_N_FLUSH] += 1;
                     }
                 }
             }
+        }
+        __syncthreads();
+        {
+            const unsigned total = s_total < (unsigned)kStage ? s_total : (unsigned)kStage;
+            if (total > 0) {
+                // ---------------------------------------------------- flush to the ring
+                const long long tf = prof ? clock64() : 0;
+                if (warp == 0 && lane < (int)p.nb) {
+                    const unsigned c = s_cnt[lane];
+                    if (p.dynamic) {
+                        if (lane == 0) atomicAdd(&p.ctl->g_push, (unsigned long long)(total + s_direct));
+                        if (lane == (int)nbm && c) atomicAdd(&p.ctl->g_clip, (unsigned long long)c);
+                    }
+                    if (c) {
+                        const unsigned sl = (hs + lane) & nbm;
+                        // returning atomic: the reserve (which also counts the children for
+                        // termination) is performed before this CTA's completion atomic
+                        const unsigned long long b = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
+                        s_base[lane] = b;
+                        if (b + c > p.cap) {  // lapping: previous occupants must be claimed
+                            const unsigned long long cl = ld_relaxed_u64(&p.bk[sl].claim.v);
+                            if (b + c - p.cap > cl) atomicOr(&p.ctl->status, kStRingOverflow);
+                        }
+                    }
+                }
+                __syncthreads();
+                for (unsigned i = tid; i < total; i += BT) {
+                    const unsigned o = s_soff[i];
+                    if (o == 0xFF) continue;  // hole left by a direct publication
+                    const unsigned sl = (hs + o) & nbm;
+                    const unsigned long long idx = s_base[o] + s_rank[i];
+                    char* sp = p.ring + ((size_t)sl * p.cap + (idx & (p.cap - 1))) * IT::kBytes;
+                    bool ok = true;
+                    if (idx >= p.cap) {  // wait for the previous lap's reader to clear it
+                        unsigned spins = 0;
+                        while (!IT::empty(sp)) {
+                            if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) {
+                                ok = false;
+                                break;
+                            }
+                        }
+                    }
+                    if (ok) IT::store(sp, s_items[i]);
+                }
+                __syncthreads();
+                if (warp == 0 && lane < (int)p.nb) {
+                    const unsigned c = s_cnt[lane];
+                    if (c) {
+                        atomicAdd(&p.bk[(hs + lane) & nbm].avail.v, (unsigned long long)c);  // publish
+                        s_cnt[lane] = 0;
+                    }
+                }
+                if (prof) {
+                    tq += clock64() - tf;
+                    s_prof[PR_N_FLUSH] += 1;
+                }
+            } else if (p.dynamic && tid == 0 && s_direct) {
+                atomicAdd(&p.ctl->g_push, (unsigned long long)s_direct);
+            }
+            if (tid == 0) {
+                c_push += total + s_direct;
+                s_total = 0;
+                s_direct = 0;
+            }
+            __syncthreads();
         }
         if (prof) {
             const long long t1 = clock64();

@@ -279,7 +279,13 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
     // the concurrently live dist arrays and mark dist accesses evict_last over
     // the fraction that fits
     p.keep_frac = 0.0f;
-    if (!(g->opts.flags & SSSP_FLAG_NO_L2_PERSIST) && g->persist_max) {
+    if (!(g->opts.flags & SSSP_FLAG_L2_PERSIST) && g->persist_max) {
+        // the driver's default set-aside (~25 MB on B200) only shrinks the normal L2
+        size_t cur = 0;
+        cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+        if (cur) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
+    }
+    if ((g->opts.flags & SSSP_FLAG_L2_PERSIST) && g->persist_max) {
         const size_t want = (size_t)g->n * sizeof(DistT) * conc;
         const size_t use = std::min(want, g->persist_max);
         size_t cur = 0;
