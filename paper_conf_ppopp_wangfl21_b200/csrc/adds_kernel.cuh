@@ -36,6 +36,9 @@
 //            Delta controller on the ring occupancy in the same step.
 //   finish   (A10) every bucket complete  <=>  quiescent.
 #pragma once
+#ifndef STAGE_MULT
+#define STAGE_MULT 4  // staging capacity = STAGE_MULT/2 * BT * EPT items
+#endif
 #include "bucket_map.h"
 #include "common.cuh"
 
@@ -344,14 +347,16 @@ constexpr size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
 template <typename DistT, int BT, int EPT, int W>
 struct Smem {
     using Raw = typename ItemT<DistT>::Raw;
-    static constexpr int kStage = 2 * BT * EPT;  // staged ring pushes before a forced flush
-    static constexpr size_t o_arc = 0;                                        // uint2[W]   arc window
-    static constexpr size_t o_items = o_arc + (size_t)W * 8;                  // Raw[kStage] staged pushes
+    // staged ring pushes of one batch (beyond this, warps publish directly)
+    // (shared memory is taken from the L1 that holds in-flight misses: keep it small)
+    static constexpr int kStage = STAGE_MULT * BT * EPT / 2;
+    static constexpr size_t o_arc = 0;                                        // (no arc window)
+    static constexpr size_t o_items = 0;                                      // Raw[kStage] staged pushes
     static constexpr size_t o_ebeg = o_items + align16((size_t)kStage * sizeof(Raw));  // u64[BT] row begin
     static constexpr size_t o_d = o_ebeg + (size_t)BT * 8;                    // DistT[BT]  item distance
     static constexpr size_t o_ld = o_d + align16((size_t)BT * sizeof(DistT)); // DistT[BT]  kept children
-    static constexpr size_t o_owner = o_ld + align16((size_t)BT * sizeof(DistT));  // u16[W] arc -> item
-    static constexpr size_t o_rank = o_owner + align16((size_t)W * 2);        // u16[kStage]
+    static constexpr size_t o_owner = o_ld + align16((size_t)BT * sizeof(DistT));  // (unused)
+    static constexpr size_t o_rank = o_owner;                                 // u16[kStage]
     static constexpr size_t o_scan = o_rank + align16((size_t)kStage * 2);    // u32[BT]
     static constexpr size_t o_lv = o_scan + align16((size_t)BT * 4);          // u32[BT] kept children
     static constexpr size_t o_soff = o_lv + align16((size_t)BT * 4);          // u8[kStage]
@@ -366,17 +371,13 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
     using L = Smem<DistT, BT, EPT, W>;
     constexpr int kStage = L::kStage;
     constexpr int kWarps = BT / 32;
-    constexpr int kPer = W / BT;      // window positions per thread in the owner scan
     constexpr unsigned long long kInf = (unsigned long long)DistInf<DistT>::value;
-    static_assert(W % BT == 0 && kPer >= 1, "window");
 
     extern __shared__ __align__(16) unsigned char smem[];
-    uint2* s_arc = (uint2*)(smem + L::o_arc);
     Raw* s_items = (Raw*)(smem + L::o_items);
     unsigned long long* s_ebeg = (unsigned long long*)(smem + L::o_ebeg);
     DistT* s_d = (DistT*)(smem + L::o_d);
     DistT* s_ld = (DistT*)(smem + L::o_ld);
-    unsigned short* s_owner = (unsigned short*)(smem + L::o_owner);
     unsigned short* s_rank = (unsigned short*)(smem + L::o_rank);
     unsigned* s_scan = (unsigned*)(smem + L::o_scan);
     unsigned* s_lv = (unsigned*)(smem + L::o_lv);
@@ -393,7 +394,6 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const unsigned lt_mask = lanemask_lt();
-    const unsigned s_arc_addr = smem_addr(s_arc);
     const unsigned nbm = p.nb - 1;
     const unsigned local_max = p.local_max < (unsigned)BT ? p.local_max : (unsigned)BT;
     unsigned long long c_vert = 0, c_edges = 0, c_push = 0, c_stale = 0, c_local = 0;  // thread 0
