@@ -43,6 +43,7 @@ WORKLOADS = {
 }
 METRIC = "GTEPS (E_dij per second) and ms/source, single-source SSSP"
 L2_BYTES = 126 * 2**20
+GATHER_PEAK_G = 280.0  # measured random L2 gather rate (tools/gather_bench.cu, this pool's B200)
 
 
 def peaks():
@@ -284,6 +285,11 @@ def run_ours(args, world, rank, local):
         # 12 B per arc relaxed (8 B {col,w} + 4 B dist gather) + 20 B per vertex expanded
         alg_bytes = (12 * E_gpu + 20 * V_gpu) / max(1, units)
         achieved = alg_bytes / (per_launch_ms / 1e3) / 1e9
+        # the bound actually binding: random 4-byte L2 accesses, one
+        # distinct line each -- a dist gather per arc, an atomic per push, and
+        # dist + row-offset + item accesses per popped item
+        rand_acc = (E_gpu + pushes + 3 * V_gpu) / max(1, units)
+        rand_rate = rand_acc / (per_launch_ms / 1e3) / 1e9
         traffic = ncu_traffic(args.config)
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
@@ -314,6 +320,10 @@ def run_ours(args, world, rank, local):
                          "frac": achieved / hbm, "traffic": traffic, "peak_kind": peak_kind,
                          "kernel": "adds_persistent_kernel", "kernel_ms_avg": per_launch_ms,
                          "alg_bytes_per_launch": alg_bytes},
+            "gather_roofline": {"bound": "l2_random_access", "achieved": rand_rate, "unit": "G accesses/s",
+                                "peak": GATHER_PEAK_G, "frac": rand_rate / GATHER_PEAK_G,
+                                "peak_source": "tools/gather_bench.cu on B200: random 4-byte gathers, "
+                                               "67 MB L2-resident array, 1184x256 threads"},
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": int(launches),

@@ -341,6 +341,60 @@ __device__ __forceinline__ unsigned bucket_of(unsigned long long nd, unsigned k,
     }
 }
 
+// --------------------------------------------------------------- claim (A4)
+// Warp-cooperative: status + head (lane 0), then the A active buckets' avail
+// gates (idle CTAs poll here, so every extra line read lands on a hot L2 slice);
+// the highest-priority bucket with published items is claimed: avail -=
+// want, give back the excess, claim += got.  Returns got (0 = none); every output
+// is warp-uniform: the claim (slot, ring index), the head snapshot and the status.
+template <typename DistT, int BT>
+__device__ unsigned claim_batch(const Params<DistT>& p, int lane, unsigned& o_slot, unsigned long long& o_idx,
+                                Head& o_head, unsigned& o_status) {
+    const unsigned nbm = p.nb - 1;
+    unsigned st = 0;
+    Head hd{0ull, 0ull};
+    if (lane == 0) {
+        st = ld_relaxed_u32(&p.ctl->status);
+        hd = ld_head(&p.ctl->head);
+    }
+    st = __shfl_sync(FULL, st, 0);
+    hd.h = __shfl_sync(FULL, hd.h, 0);
+    hd.meta = __shfl_sync(FULL, hd.meta, 0);
+    o_status = st;
+    o_head = hd;
+    if (st) return 0;
+    const unsigned hs = meta_hs(hd.meta), A = meta_A(hd.meta);
+    long long av = 0;
+    if (lane < (int)A) av = (long long)ld_relaxed_u64(&p.bk[(hs + lane) & nbm].avail.v);
+    unsigned mask = __ballot_sync(FULL, av > 0);
+    while (mask) {
+        const int f = __ffs(mask) - 1;
+        unsigned g32 = 0, sl32 = 0;
+        unsigned long long ix = 0;
+        if (lane == f) {
+            const unsigned sl = (hs + f) & nbm;
+            long long want = av >> p.share_shift;
+            if (want < (long long)p.batch_min) want = p.batch_min;
+            if (want > BT) want = BT;
+            unsigned long long* avp = &p.bk[sl].avail.v;
+            const long long old = (long long)atomicAdd(avp, (unsigned long long)(-want));
+            const long long g = old <= 0 ? 0 : (old < want ? old : want);
+            if (g < want) atomicAdd(avp, (unsigned long long)(want - g));
+            if (g > 0) ix = atomicAdd(&p.bk[sl].claim.v, (unsigned long long)g);
+            g32 = (unsigned)g;
+            sl32 = sl;
+        }
+        g32 = __shfl_sync(FULL, g32, f);
+        if (g32) {
+            o_idx = __shfl_sync(FULL, ix, f);
+            o_slot = __shfl_sync(FULL, sl32, f);
+            return g32;
+        }
+        mask &= mask - 1;
+    }
+    return 0;
+}
+
 // --------------------------------------------------------------- shared memory
 constexpr size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
 
@@ -426,61 +480,28 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
             // -------------------------------------------------------- claim
             if (warp == 0) {
                 int cmd = CMD_IDLE;
-                // status + head (lane 0), then only the A active buckets' avail gates:
-                // idle CTAs poll here, so every extra line read lands on a hot L2 slice
-                unsigned st = 0;
-                Head hd{0ull, 0ull};
-                if (lane == 0) {
-                    st = ld_relaxed_u32(&p.ctl->status);
-                    hd = ld_head(&p.ctl->head);
-                }
-                st = __shfl_sync(FULL, st, 0);
-                hd.h = __shfl_sync(FULL, hd.h, 0);
-                hd.meta = __shfl_sync(FULL, hd.meta, 0);
-                const unsigned hs = meta_hs(hd.meta), A = meta_A(hd.meta);
-                long long av = 0;
-                if (lane < (int)A && !st) av = (long long)ld_relaxed_u64(&p.bk[(hs + lane) & nbm].avail.v);
+                unsigned sl = 0, st = 0;
+                unsigned long long idx = 0;
+                Head hd;
+                const unsigned g = claim_batch<DistT, BT>(p, lane, sl, idx, hd, st);
                 if (st) {
                     cmd = CMD_EXIT;
-                } else {
-                    unsigned mask = __ballot_sync(FULL, av > 0);
-                    while (mask) {  // higher-priority buckets first
-                        const int f = __ffs(mask) - 1;
-                        unsigned g32 = 0;
-                        if (lane == f) {
-                            const unsigned sl = (hs + f) & nbm;
-                            long long want = av >> p.share_shift;
-                            if (want < (long long)p.batch_min) want = p.batch_min;
-                            if (want > BT) want = BT;
-                            unsigned long long* avp = &p.bk[sl].avail.v;
-                            const long long old = (long long)atomicAdd(avp, (unsigned long long)(-want));
-                            const long long g = old <= 0 ? 0 : (old < want ? old : want);
-                            if (g < want) atomicAdd(avp, (unsigned long long)(want - g));
-                            if (g > 0) {
-                                s_idx = atomicAdd(&p.bk[sl].claim.v, (unsigned long long)g);
-                                s_got = (unsigned)g;
-                                s_slot = sl;
-                                s_head = hd;
-                            }
-                            g32 = (unsigned)g;
-                        }
-                        g32 = __shfl_sync(FULL, g32, f);
-                        if (g32) {
-                            cmd = CMD_WORK;
-                            break;
-                        }
-                        mask &= mask - 1;
-                    }
-                    if (cmd != CMD_WORK) {
-                        if (try_advance<DistT>(p, hd, lane)) {
-                            cmd = CMD_EXIT;
-                        } else if (lane == 0) {
-                            if (globaltimer() - p.ctl->t_start > p.timeout_ns) atomicOr(&p.ctl->status, kStTimeout);
-                            backoff = backoff ? (backoff * 2 < p.max_backoff_ns ? backoff * 2 : p.max_backoff_ns) : 32;
-                            __nanosleep(backoff);
-                        }
-                    } else if (lane == 0) {
+                } else if (g) {
+                    cmd = CMD_WORK;
+                    if (lane == 0) {
+                        s_got = g;
+                        s_slot = sl;
+                        s_idx = idx;
+                        s_head = hd;
                         backoff = 0;
+                    }
+                } else {
+                    if (try_advance<DistT>(p, hd, lane)) {
+                        cmd = CMD_EXIT;
+                    } else if (lane == 0) {
+                        if (globaltimer() - p.ctl->t_start > p.timeout_ns) atomicOr(&p.ctl->status, kStTimeout);
+                        backoff = backoff ? (backoff * 2 < p.max_backoff_ns ? backoff * 2 : p.max_backoff_ns) : 32;
+                        __nanosleep(backoff);
                     }
                 }
                 if (lane == 0) s_cmd = cmd;
