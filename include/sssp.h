@@ -106,7 +106,7 @@ typedef struct sssp_options {
     uint32_t waste_lo_permille;/* Delta may grow only while the recent re-expansion share is below this
                                   (default 450 = 45%) */
     uint32_t waste_hi_permille;/* Delta shrinks (not below its clip floor) while the share is above this
-                                  (default 500 = 50%, i.e. ~2x Dijkstra's vertex work) */
+                                  (default 600 = 60%, i.e. ~2.5x Dijkstra's vertex work) */
     uint32_t period_us;        /* periodic controller step (default 20 us; head switches also step) */
     uint32_t delta_heuristic;  /* initial-Delta heuristic when delta_init == 0 ("a heuristic similar
                                   to the one described in Section 4.3"): SSSP_DELTA_H_RING_SPAN (default:
@@ -138,7 +138,13 @@ typedef struct sssp_options {
     uint32_t algorithm;        /* SSSP_ALGO_ADDS (default) or SSSP_ALGO_NEAR_FAR: the paper's comparison
                                   system as an ablation -- 2 buckets, static Delta (default the
                                   Near-Far rule C*W/D), bulk-synchronous double-buffered piles */
-    uint32_t reserved2[3];
+    uint32_t split_degree;     /* hub splitting (§8(a) A5 "CTA/edge-chunk bins"): an expanded vertex with
+                                  more out-arcs than this is processed by its CTA for the first
+                                  split_degree arcs while the rest is published as split_degree-arc
+                                  chunks that idle CTAs claim before bucket items (charged to the
+                                  vertex's bucket, so the head cannot pass it early); 0 = auto
+                                  (8 x CTA size), UINT32_MAX = off */
+    uint32_t reserved2[2];
 } sssp_options;
 
 typedef struct sssp_stats {

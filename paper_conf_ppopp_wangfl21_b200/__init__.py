@@ -72,7 +72,7 @@ class sssp_options(ctypes.Structure):
         ("batch_min", ctypes.c_uint32), ("timeout_ms", ctypes.c_uint32), ("trace_capacity", ctypes.c_uint32),
         ("active_init", ctypes.c_uint32), ("local_max", ctypes.c_uint32), ("max_backoff_ns", ctypes.c_uint32),
         ("startup_permille", ctypes.c_uint32), ("concurrent_sources", ctypes.c_uint32),
-        ("algorithm", ctypes.c_uint32), ("reserved2", ctypes.c_uint32 * 3),
+        ("algorithm", ctypes.c_uint32), ("split_degree", ctypes.c_uint32), ("reserved2", ctypes.c_uint32 * 2),
     ]
 
 

@@ -76,6 +76,9 @@ struct Params {
     unsigned waste_lo, waste_hi;  // permille
     unsigned long long period_ns;
     unsigned long long startup_first;  // no Delta growth before this many first expansions
+    SplitTask* tasks;          // hub-split chunk queue (counters in bk[kSplitQ])
+    unsigned long long tcap;   // entries, power of two
+    unsigned split_deg;        // split vertices with more arcs than this (0 = off)
     unsigned k_max;
     unsigned long long timeout_ns;
 };
@@ -103,7 +106,7 @@ __device__ __forceinline__ long long warp_sum_s64(long long x) {
 // steps) since the last Delta change; a change needs since >= settle (a quarter
 // of that for growth while the re-expansion share is below waste_lo / 8).
 struct CtlDecision {
-    unsigned k, A, flo, since;
+    unsigned k, A, flo, since, ceil;
     bool changed;
     unsigned flags;  // decision inputs, recorded in the trace: 1 low, 2 high, 4 beyond, 8 wasteful,
                      // 16 frugal, 32 clipping, 64 waste known, 128 progressed, 256 settled
@@ -114,9 +117,14 @@ struct CtlDecision {
 // over the recent window.  clip = share of recent pushes that were clipped.
 template <typename DistT>
 __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, unsigned flo, unsigned since,
-                              long long total, long long tail, long long win, unsigned waste, bool waste_known,
-                              unsigned clip, bool clip_known, unsigned ratio_x100, bool progressed) {
-    CtlDecision d{k, A, flo, since + 1, false, 0u};
+                              unsigned ceil, bool head_switch, long long total, long long tail, long long win, unsigned waste,
+                              bool waste_known, unsigned clip, bool clip_known, unsigned ratio_x100,
+                              bool progressed) {
+    // since = [0,8) controller steps, [8,16) head switches since the last change
+    unsigned steps = since & 0xffu, hsw = (since >> 8) & 0xffu;
+    steps = steps < 255u ? steps + 1 : 255u;
+    if (head_switch && hsw < 255u) ++hsw;
+    CtlDecision d{k, A, flo, steps | (hsw << 8), ceil, false, 0u};
     if (!p.dynamic) return d;
     const unsigned long long util = ((unsigned long long)(win > 0 ? win : 0) * p.avg_deg_x16) >> 4;
     const unsigned long long T = p.resident_threads;
@@ -126,29 +134,38 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
     // waste: recent re-expansions high AND the run as a whole already above 2x
     // (both need the start-up gate: early samples are tiny and noisy)
     const bool wasteful = progressed && waste_known && waste > p.waste_hi && ratio_x100 > 200;
-    // frugal: recent and cumulative re-expansion both low
-    // (no growth during the start-up transient: the first frontier is always small)
+    // frugal: recent re-expansion low, and either the run as a whole is below 1.5x
+    // or the recent share is below half the growth limit (a bad start-up must not
+    // block growth for the rest of the run)
     // (an unmeasurable waste -- too few expansions in the window -- means the run
     // is crawling: growth is allowed once the start-up gate is open)
-    const bool frugal = (!waste_known || waste < p.waste_lo) && ratio_x100 < 150 && progressed;
+    const bool frugal = (!waste_known || waste < p.waste_lo) &&
+                        (ratio_x100 < 150 || !waste_known || waste * 2 < p.waste_lo) && progressed;
     const bool clipping = (total >= 64 && tail * 100 >= (long long)p.clip_pct * total) || (clip_known && clip >= 500);
+    // settled: enough steps AND the head has switched twice since the last
+    // change, so the ring has turned over and the items placed under the previous
+    // Delta -- whose slots now mix priorities -- are no longer what the
+    // waste signal measures (without this, shrinks fed on their own mixing waste)
+    const bool turned = hsw >= 2;
     d.flags = (low ? 1u : 0u) | (high ? 2u : 0u) | (beyond ? 4u : 0u) | (wasteful ? 8u : 0u) |
               (frugal ? 16u : 0u) | (clipping ? 32u : 0u) | (waste_known ? 64u : 0u) | (progressed ? 128u : 0u) |
-              (d.since >= p.settle ? 256u : 0u);
-    if (clipping && k < p.k_max && d.since >= 2) {
+              (steps >= p.settle && turned ? 256u : 0u);
+    if (clipping && k < p.k_max && steps >= 2) {
         d.k = k + 1;  // clipping: raise Delta and its lower bound
         d.flo = d.k;
+        if (d.ceil <= d.k) d.ceil = 0xffu;  // the clip bound overrides the waste ceiling
         d.changed = true;
-    } else if (d.since >= p.settle) {
+    } else if (steps >= p.settle && turned) {
         if (wasteful && k > flo) {
             d.k = k - 1;
+            d.ceil = k;  // hysteresis: do not grow back into a Delta measured wasteful
             d.changed = true;
-        } else if (low && frugal && beyond && k < p.k_max) {
+        } else if (low && frugal && beyond && k < p.k_max && k + 1 < ceil) {
             d.k = k + 1;
             d.changed = true;
         }
-    } else if (d.since * 4 >= p.settle && low && frugal && beyond && (!waste_known || waste * 8 < p.waste_lo) &&
-               k < p.k_max) {
+    } else if (steps * 4 >= p.settle && turned && low && frugal && beyond && (!waste_known || waste * 8 < p.waste_lo) &&
+               k < p.k_max && k + 1 < ceil) {
         d.k = k + 1;  // essentially no re-expansion yet: grow with a quarter of the settling time
         d.changed = true;
     }
@@ -157,7 +174,7 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
     // under-utilised, work waits beyond the window and almost nothing is
     // re-expanded; back to fewer when wasteful or busy
     if (p.adapt_active) {
-        if (low && beyond && waste_known && waste < p.waste_lo / 4 && ratio_x100 < 115 && d.since >= p.settle &&
+        if (low && beyond && waste_known && waste < p.waste_lo / 4 && ratio_x100 < 115 && steps >= p.settle &&
             A < p.nb)
             d.A = A + 1;
         else if ((wasteful || high) && A > 1)
@@ -274,12 +291,12 @@ __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lan
     bool known, cknown;
     const unsigned waste = recent_waste(p, known);
     const unsigned clip = recent_clip(p, cknown);
-    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), total, tail, win, waste, known,
-                                 clip, cknown, cumulative_ratio(p),
+    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), meta_ceil(hd.meta), true, total, tail, win, waste,
+                                 known, clip, cknown, cumulative_ratio(p),
                                  ld_relaxed_u64(&p.ctl->g_first) >= p.startup_first ||
                                      ld_relaxed_u32(&p.ctl->head_switches) >= 32u);
     const Head nhd{rehead(hd.h + o, k, d.k),
-                   pack_meta((hs + o) & (nb - 1), d.k, d.A, d.flo, d.since > 0xffff ? 0xffff : d.since)};
+                   pack_meta((hs + o) & (nb - 1), d.k, d.A, d.flo, d.since, d.ceil)};
     commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 1u, d.flags);
     return false;
 }
@@ -299,11 +316,11 @@ __device__ void periodic_step(const Params<DistT>& p, const int lane) {
     bool known, cknown;
     const unsigned waste = recent_waste(p, known);
     const unsigned clip = recent_clip(p, cknown);
-    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), total, tail, win, waste, known,
-                                 clip, cknown, cumulative_ratio(p),
+    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), meta_ceil(hd.meta), false, total, tail, win, waste,
+                                 known, clip, cknown, cumulative_ratio(p),
                                  ld_relaxed_u64(&p.ctl->g_first) >= p.startup_first ||
                                      ld_relaxed_u32(&p.ctl->head_switches) >= 32u);
-    const Head nhd{rehead(hd.h, k, d.k), pack_meta(hs, d.k, d.A, d.flo, d.since > 0xffff ? 0xffff : d.since)};
+    const Head nhd{rehead(hd.h, k, d.k), pack_meta(hs, d.k, d.A, d.flo, d.since, d.ceil)};
     commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 2u, d.flags);
 }
 
@@ -347,9 +364,15 @@ __device__ __forceinline__ unsigned bucket_of(unsigned long long nd, unsigned k,
 // the highest-priority bucket with published items is claimed: avail -=
 // want, give back the excess, claim += got.  Returns got (0 = none); every output
 // is warp-uniform: the claim (slot, ring index), the head snapshot and the status.
+//
+// Hub-split chunks come first (lane 31 polls their gate in the same round trip):
+// they are the unfinished rest of an already-claimed item, usually of the head
+// bucket, which cannot complete before they do.  A chunk claim returns 1 with
+// o_task set and o_idx = the chunk's queue index.
 template <typename DistT, int BT>
 __device__ unsigned claim_batch(const Params<DistT>& p, int lane, unsigned& o_slot, unsigned long long& o_idx,
-                                Head& o_head, unsigned& o_status) {
+                                Head& o_head, unsigned& o_status, bool& o_task) {
+    o_task = false;
     const unsigned nbm = p.nb - 1;
     unsigned st = 0;
     Head hd{0ull, 0ull};
@@ -364,8 +387,29 @@ __device__ unsigned claim_batch(const Params<DistT>& p, int lane, unsigned& o_sl
     o_head = hd;
     if (st) return 0;
     const unsigned hs = meta_hs(hd.meta), A = meta_A(hd.meta);
-    long long av = 0;
+    long long av = 0, tv = 0;
     if (lane < (int)A) av = (long long)ld_relaxed_u64(&p.bk[(hs + lane) & nbm].avail.v);
+    if (p.split_deg && lane == 31) tv = (long long)ld_relaxed_u64(&p.bk[kSplitQ].avail.v);
+    if (__shfl_sync(FULL, tv, 31) > 0) {
+        unsigned got = 0;
+        unsigned long long ix = 0;
+        if (lane == 31) {
+            unsigned long long* avp = &p.bk[kSplitQ].avail.v;
+            const long long old = (long long)atomicAdd(avp, (unsigned long long)(-1ll));
+            if (old > 0) {
+                ix = atomicAdd(&p.bk[kSplitQ].claim.v, 1ull);
+                got = 1;
+            } else {
+                atomicAdd(avp, 1ull);
+            }
+        }
+        if (__shfl_sync(FULL, got, 31)) {
+            o_idx = __shfl_sync(FULL, ix, 31);
+            o_slot = 0;
+            o_task = true;
+            return 1;
+        }
+    }
     unsigned mask = __ballot_sync(FULL, av > 0);
     while (mask) {
         const int f = __ffs(mask) - 1;
@@ -395,10 +439,48 @@ __device__ unsigned claim_batch(const Params<DistT>& p, int lane, unsigned& o_sl
     return 0;
 }
 
+// --------------------------------------------------------------- hub split (A5)
+// Publish arcs [S, deg) of vertex v (expanded at distance d, row begins at b) as
+// chunks of S arcs; the caller processes the first S itself.  The chunks are
+// charged to the item's ring slot BEFORE they become claimable, so the bucket
+// stays incomplete (the head cannot pass it) until every chunk is done.
+template <typename DistT>
+__device__ unsigned spawn_chunks(const Params<DistT>& p, unsigned v, unsigned long long d, unsigned long long b,
+                                 unsigned deg, unsigned slot) {
+    const unsigned S = p.split_deg;
+    const unsigned extra = (deg - 1) / S;
+    atomicAdd(&p.bk[slot].local.v, (unsigned long long)extra);
+    const unsigned long long t0 = atomicAdd(&p.bk[kSplitQ].reserve.v, (unsigned long long)extra);
+    if (t0 + extra > p.tcap && t0 + extra - p.tcap > ld_relaxed_u64(&p.bk[kSplitQ].claim.v)) {
+        atomicOr(&p.ctl->status, kStRingOverflow);  // would lap an unclaimed chunk: regrow and re-run
+        return S;
+    }
+    for (unsigned c = 1; c <= extra; ++c) {
+        const unsigned long long idx = t0 + c - 1;
+        SplitTask* tp = p.tasks + (idx & (p.tcap - 1));
+        if (idx >= p.tcap) {  // the previous lap's occupant is claimed: wait for its reader to clear it
+            unsigned spins = 0;
+            while (ld_relaxed_u32(&tp->len) != 0)
+                if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) return S;
+        }
+        tp->beg = b + (unsigned long long)c * S;
+        tp->d = d;
+        tp->v = v;
+        tp->slot = slot;
+    }
+    __threadfence();  // payloads before their len markers
+    for (unsigned c = 1; c <= extra; ++c) {
+        const unsigned rest = deg - c * S;
+        st_relaxed_u32(&p.tasks[(t0 + c - 1) & (p.tcap - 1)].len, rest < S ? rest : S);
+    }
+    atomicAdd(&p.bk[kSplitQ].avail.v, (unsigned long long)extra);
+    return S;
+}
+
 // --------------------------------------------------------------- shared memory
 constexpr size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
 
-template <typename DistT, int BT, int EPT, int W>
+template <typename DistT, int BT, int EPT>
 struct Smem {
     using Raw = typename ItemT<DistT>::Raw;
     // staged ring pushes of one batch (beyond this, warps publish directly)
@@ -418,11 +500,15 @@ struct Smem {
 };
 
 // --------------------------------------------------------------- kernel
-template <typename DistT, int BT, int EPT, int W, bool kF>
-__global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Params<DistT> p) {
+// BT threads per CTA, EPT arcs per thread per round, MINB CTAs per SM (register
+// budget 65536 / (MINB * BT)), PIPE: the arc loads of a warp's next round are
+// issued before the current round's gathers/atomics (software pipeline: one
+// fewer dependent L2/HBM trip per round), kF: float32 weights (NEXT-3).
+template <typename DistT, int BT, int EPT, int MINB, bool PIPE, bool kF>
+__global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<DistT> p) {
     using IT = ItemT<DistT>;
     using Raw = typename IT::Raw;
-    using L = Smem<DistT, BT, EPT, W>;
+    using L = Smem<DistT, BT, EPT>;
     constexpr int kStage = L::kStage;
     constexpr int kWarps = BT / 32;
     constexpr unsigned long long kInf = (unsigned long long)DistInf<DistT>::value;
@@ -440,7 +526,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
     __shared__ unsigned s_cnt[kMaxBuckets];
     __shared__ unsigned long long s_base[kMaxBuckets];
     __shared__ unsigned s_wsum[kWarps];
-    __shared__ unsigned s_total, s_E, s_got, s_slot, s_lnext, s_direct;
+    __shared__ unsigned s_total, s_E, s_got, s_slot, s_lnext, s_direct, s_task;
     __shared__ int s_cmd;
     __shared__ unsigned long long s_idx;
     __shared__ Head s_head;
@@ -470,7 +556,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
 
     for (;;) {
         unsigned got, slot;
-        bool from_ring;
+        bool from_ring, is_task = false;
         if (prof) t0 = clock64();
         if (have_local) {
             got = have_local;
@@ -483,7 +569,8 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                 unsigned sl = 0, st = 0;
                 unsigned long long idx = 0;
                 Head hd;
-                const unsigned g = claim_batch<DistT, BT>(p, lane, sl, idx, hd, st);
+                bool tk;
+                const unsigned g = claim_batch<DistT, BT>(p, lane, sl, idx, hd, st, tk);
                 if (st) {
                     cmd = CMD_EXIT;
                 } else if (g) {
@@ -493,6 +580,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                         s_slot = sl;
                         s_idx = idx;
                         s_head = hd;
+                        s_task = tk ? 1u : 0u;
                         backoff = 0;
                     }
                 } else {
@@ -519,6 +607,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
             got = s_got;
             slot = s_slot;
             from_ring = true;
+            is_task = s_task != 0;
         }
 
         // CTA-local continuation only in the latency regime (small batches = scarce
@@ -531,7 +620,29 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
         const unsigned hs = meta_hs(hd.meta), k = meta_k(hd.meta);
         unsigned deg = 0;
         bool live = false, first = false;
-        if (tid < (int)got) {
+        if (is_task) {
+            // a hub-split chunk: one vertex, len arcs, charged to the slot it carries
+            if (tid == 0) {
+                SplitTask* tp = p.tasks + (s_idx & (p.tcap - 1));
+                unsigned len, spins = 0;
+                s_slot = 0;
+                while ((len = ld_acquire_u32(&tp->len)) == 0)
+                    if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;
+                if (len) {
+                    const unsigned long long b = __ldcg(&tp->beg), d = __ldcg(&tp->d);
+                    const unsigned v = __ldcg(&tp->v);
+                    s_slot = __ldcg(&tp->slot);
+                    st_relaxed_u32(&tp->len, 0u);  // clear behind the read
+                    const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
+                    if (cur >= d) {  // stale chunks (v improved since) are dropped
+                        deg = len;
+                        s_ebeg[0] = b;
+                        s_d[0] = (DistT)d;
+                        live = true;
+                    }
+                }
+            }
+        } else if (tid < (int)got) {
             uint32_t v;
             unsigned long long d;
             bool loaded = true;
@@ -561,6 +672,7 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                         const unsigned bit = 1u << (v & 31);
                         first = (atomicOr(p.expanded + (v >> 5), bit) & bit) == 0;
                     }
+                    if (p.split_deg && deg > p.split_deg) deg = spawn_chunks(p, v, d, b, deg, slot);
                 }
             }
         }
@@ -595,9 +707,11 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
         __syncthreads();
         s_scan[tid] = x - deg + s_wsum[warp];
         const unsigned E = s_E;
+        if (is_task) slot = s_slot;
+        const int nexp = is_task ? 0 : nlive;  // a chunk is not a vertex expansion
         if (tid == 0) {
-            c_vert += nlive;
-            c_stale += got - nlive;
+            c_vert += nexp;
+            if (!is_task) c_stale += got - nlive;
             c_edges += E;
         }
         if (prof) {
@@ -621,14 +735,11 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
             const unsigned slice = (per + 31) / 32 * 32;  // small batches spread over many warps
             const unsigned wb = warp * slice;
             const unsigned we = (wb + slice) < E ? (wb + slice) : E;
-            for (unsigned base = wb; base < we; base += 32 * EPT) {
-                unsigned own[EPT];
-                uint2 a[EPT];
-                unsigned long long nd[EPT];
-                bool push[EPT];
-                DistT cur[EPT];
+            // owner of each arc (largest i with scan[i] <= e, binary search in shared
+            // memory) and its coalesced {col, w} load
+            auto fetch = [&](unsigned base, unsigned (&own)[EPT], uint2 (&a)[EPT]) {
 #pragma unroll
-                for (int j = 0; j < EPT; ++j) {  // owner = largest i with scan[i] <= e
+                for (int j = 0; j < EPT; ++j) {
                     const unsigned e = base + j * 32 + lane;
                     unsigned lo = 0, hi = got - 1;
                     if (e < we) {
@@ -643,13 +754,19 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {  // EPT independent arc loads in flight
                     const unsigned e = base + j * 32 + lane;
-                    if (e < we) {
-                        a[j] = ld_stream_u2(p.adj + s_ebeg[own[j]] + (e - s_scan[own[j]]), pol_stream);
-                        nd[j] = relax_sum<kF>((unsigned long long)s_d[own[j]], a[j].y);
-                    } else {
-                        a[j] = make_uint2(0u, 0u);
-                        nd[j] = kInf;
-                    }
+                    a[j] = e < we ? ld_stream_u2(p.adj + s_ebeg[own[j]] + (e - s_scan[own[j]]), pol_stream)
+                                  : make_uint2(0u, 0u);
+                }
+            };
+            // relax + push of one round whose arcs are loaded
+            auto body = [&](const unsigned base, const unsigned (&own)[EPT], const uint2 (&a)[EPT]) {
+                unsigned long long nd[EPT];
+                bool push[EPT];
+                DistT cur[EPT];
+#pragma unroll
+                for (int j = 0; j < EPT; ++j) {
+                    const unsigned e = base + j * 32 + lane;
+                    nd[j] = e < we ? relax_sum<kF>((unsigned long long)s_d[own[j]], a[j].y) : kInf;
                 }
 #pragma unroll
                 for (int j = 0; j < EPT; ++j)  // EPT independent L2 gathers in flight
@@ -752,6 +869,31 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
                         }
                     }
                 }
+            };
+            if (PIPE && we > wb + 32 * EPT) {
+                // software pipeline: round r+1's owners and arc loads are issued before
+                // round r's gathers and atomics
+                unsigned own_n[EPT];
+                uint2 a_n[EPT];
+                fetch(wb, own_n, a_n);
+                for (unsigned base = wb; base < we; base += 32 * EPT) {
+                    unsigned own[EPT];
+                    uint2 a[EPT];
+#pragma unroll
+                    for (int j = 0; j < EPT; ++j) {
+                        own[j] = own_n[j];
+                        a[j] = a_n[j];
+                    }
+                    if (base + 32 * EPT < we) fetch(base + 32 * EPT, own_n, a_n);
+                    body(base, own, a);
+                }
+            } else {
+                for (unsigned base = wb; base < we; base += 32 * EPT) {
+                    unsigned own[EPT];
+                    uint2 a[EPT];
+                    fetch(base, own, a);
+                    body(base, own, a);
+                }
             }
         }
         __syncthreads();
@@ -841,8 +983,8 @@ __global__ void __launch_bounds__(BT, 1024 / BT) adds_persistent_kernel(const Pa
         if (p.dynamic && warp == 0) {
             unsigned run_ctl = 0;
             if (lane == 0) {
-                if (nlive) {
-                    atomicAdd(&p.ctl->g_exp, (unsigned long long)nlive);
+                if (nexp) {
+                    atomicAdd(&p.ctl->g_exp, (unsigned long long)nexp);
                     atomicAdd(&p.ctl->g_first, (unsigned long long)nfirst);
                 }
                 if (kept) atomicAdd(&p.ctl->g_push, (unsigned long long)kept);

@@ -52,6 +52,7 @@ __global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned s
         expanded[i] = 0u;
     if (blockIdx.x == 0) {
         const unsigned t = threadIdx.x;
+        if (t == kSplitQ) bk[t].reserve.v = bk[t].avail.v = bk[t].claim.v = bk[t].done.v = bk[t].local.v = 0;
         if (t < kMaxBuckets) {
             bk[t].reserve.v = 0;
             bk[t].avail.v = 0;

@@ -42,6 +42,21 @@ struct BucketCtl {
     Counter done;     // items whose processing completed           = CWC
     Counter local;    // items kept CTA-local (never stored in the ring) charged to this bucket
 };
+// Hub-split chunk (§8(a) A5): arcs [beg, beg + len) of vertex v expanded at
+// distance d, charged to ring slot `slot` (its `local` counter was raised when the
+// chunk was made; completing the chunk raises `done`).  len == 0 marks an empty
+// entry: the producer stores the payload, fences, then stores len; the consumer
+// spins on len (acquire), reads, and clears it.  Queue counters live in
+// BucketCtl[kSplitQ] (reserve / avail / claim, the bucket-ring protocol).
+struct alignas(32) SplitTask {
+    unsigned long long beg;
+    unsigned long long d;
+    unsigned v;
+    unsigned len;
+    unsigned slot;
+    unsigned pad_;
+};
+constexpr uint32_t kSplitQ = kMaxBuckets;  // index of the split queue's counters
 // In flight for bucket b = reserve + local - done.  The bucket is complete when
 // that is 0, and the run is finished when every bucket is complete
 // (exact quiescence, reading R11 of P:182): children are always counted (reserve
@@ -51,23 +66,25 @@ struct BucketCtl {
 //   h    : absolute number of the head bucket (units of Delta = 2^k)
 //   meta : [0,8) hs = ring slot of the head  [8,16) k = log2 Delta
 //          [16,24) A = active buckets        [24,32) floor of k (clip bound)
-//          [32,48) head switches since the last Delta change
+//          [32,48) controller steps / head switches since the last Delta change
+//          [48,56) ceiling of k: a k found wasteful is not grown into again (0xff = none)
 struct alignas(16) Head {
     unsigned long long h;
     unsigned long long meta;
 };
 
 __host__ __device__ __forceinline__ unsigned long long pack_meta(unsigned hs, unsigned k, unsigned A,
-                                                                 unsigned flo, unsigned since) {
+                                                                 unsigned flo, unsigned since, unsigned ceil = 0xffu) {
     return (unsigned long long)(hs & 0xff) | ((unsigned long long)(k & 0xff) << 8) |
            ((unsigned long long)(A & 0xff) << 16) | ((unsigned long long)(flo & 0xff) << 24) |
-           ((unsigned long long)(since & 0xffff) << 32);
+           ((unsigned long long)(since & 0xffff) << 32) | ((unsigned long long)(ceil & 0xff) << 48);
 }
 __host__ __device__ __forceinline__ unsigned meta_hs(unsigned long long m) { return (unsigned)(m & 0xff); }
 __host__ __device__ __forceinline__ unsigned meta_k(unsigned long long m) { return (unsigned)((m >> 8) & 0xff); }
 __host__ __device__ __forceinline__ unsigned meta_A(unsigned long long m) { return (unsigned)((m >> 16) & 0xff); }
 __host__ __device__ __forceinline__ unsigned meta_floor(unsigned long long m) { return (unsigned)((m >> 24) & 0xff); }
 __host__ __device__ __forceinline__ unsigned meta_since(unsigned long long m) { return (unsigned)((m >> 32) & 0xffff); }
+__host__ __device__ __forceinline__ unsigned meta_ceil(unsigned long long m) { return (unsigned)((m >> 48) & 0xff); }
 
 struct TraceEntry {  // mirrors sssp_trace_entry
     unsigned long long time_ns, head, pending_total, pending_window, pending_tail;
@@ -115,6 +132,14 @@ __device__ __forceinline__ long long ld_relaxed_s64(const long long* p) {
     long long v;
     asm volatile("ld.relaxed.gpu.global.s64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
+}
+__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed_u32(unsigned* p, unsigned v) {
+    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 __device__ __forceinline__ unsigned ld_relaxed_u32(const unsigned* p) {
     unsigned v;

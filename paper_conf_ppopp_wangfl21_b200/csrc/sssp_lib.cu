@@ -7,6 +7,7 @@
 #include <cmath>
 #include <cstdio>
 #include <cstring>
+#include <cstdlib>
 #include <string>
 #include <vector>
 
@@ -71,6 +72,8 @@ struct Workspace {
     DevBuf dist;        // 8n bytes (serves 32- and 64-bit distances)
     DevBuf ring;        // nb * cap * item bytes
     DevBuf bk, ctl, trace, expanded;
+    DevBuf tasks;                   // hub-split chunk queue (SplitTask[tcap])
+    unsigned long long tcap = 0;
     unsigned long long cap = 0;
     int ring_item_bytes = 0;
     unsigned trace_alloc = 0;
@@ -88,6 +91,7 @@ struct Workspace {
         ctl.release();
         trace.release();
         expanded.release();
+        tasks.release();
         nf_piles.release();
         nf_cnt.release();
         if (h_ctl) cudaFreeHost(h_ctl);
@@ -162,14 +166,27 @@ struct KVariant {
     void* fn;
     size_t smem;
 };
-template <typename DistT, int BT, bool kF = false>
+template <typename DistT, int BT, bool kF = false, int EPT = 4, int MINB = 1024 / BT, bool PIPE = false>
 KVariant kvar() {
-    constexpr int W = BT >= 1024 ? 4096 : (BT >= 256 ? 2048 : 1024);
-    return KVariant{(void*)adds_persistent_kernel<DistT, BT, 4, W, kF>, Smem<DistT, BT, 4, W>::bytes};
+    return KVariant{(void*)adds_persistent_kernel<DistT, BT, EPT, MINB, PIPE, kF>, Smem<DistT, BT, EPT>::bytes};
+}
+// SSSP_KVAR (experiments): 0 default; 1 pipelined 512x2/SM EPT 4; 2 pipelined 512x1/SM EPT 8;
+// 3 pipelined 1024x1/SM EPT 4; 4 pipelined 512x1/SM EPT 4; 5 plain 512x1/SM EPT 8;
+// 6 pipelined 256x2/SM EPT 8
+static int kvar_env() {
+    const char* e = std::getenv("SSSP_KVAR");
+    return e ? std::atoi(e) : 0;
 }
 KVariant persistent_variant(int bits, int bt, bool f32) {
     if (f32) return bt == 256 ? kvar<uint32_t, 256, true>() : kvar<uint32_t, 512, true>();
+    const int kv = kvar_env();
     if (bits == 32) {
+        if (kv == 1) return kvar<uint32_t, 512, false, 4, 2, true>();
+        if (kv == 2) return kvar<uint32_t, 512, false, 8, 1, true>();
+        if (kv == 3) return kvar<uint32_t, 1024, false, 4, 1, true>();
+        if (kv == 4) return kvar<uint32_t, 512, false, 4, 1, true>();
+        if (kv == 5) return kvar<uint32_t, 512, false, 8, 1, false>();
+        if (kv == 6) return kvar<uint32_t, 256, false, 8, 2, true>();
         if (bt == 128) return kvar<uint32_t, 128>();
         if (bt == 512) return kvar<uint32_t, 512>();
         if (bt == 1024) return kvar<uint32_t, 1024>();
@@ -198,6 +215,27 @@ sssp_status ensure_ring(sssp_graph* g, Workspace& w, int item_bytes, unsigned lo
     return SSSP_OK;
 }
 
+unsigned split_degree(const sssp_graph* g, unsigned bt) {
+    if (g->opts.split_degree == 0xFFFFFFFFu) return 0u;
+    return g->opts.split_degree ? g->opts.split_degree : 8u * bt;
+}
+
+// Hub-split chunk queue: enough entries for every arc of the graph in chunks of
+// the smallest auto split degree (8 x 128), twice; doubled on overflow.
+sssp_status ensure_tasks(sssp_graph* g, Workspace& w, unsigned long long tcap) {
+    if (w.tasks.p && w.tcap == tcap) return SSSP_OK;
+    w.tasks.release();
+    const size_t bytes = (size_t)tcap * sizeof(SplitTask);
+    CK(cudaMalloc(&w.tasks.p, bytes), "allocating the split-chunk queue");
+    w.tasks.bytes = bytes;
+    CK(cudaMemset(w.tasks.p, 0, bytes), "clearing the split-chunk queue");
+    w.tcap = tcap;
+    return SSSP_OK;
+}
+unsigned long long default_tcap(const sssp_graph* g) {
+    return next_pow2(std::max<unsigned long long>(4096ull, 2ull * g->m / 1024ull));
+}
+
 sssp_status ensure_trace(sssp_graph* g, Workspace& w) {
     if (!(g->opts.flags & SSSP_FLAG_TRACE)) return SSSP_OK;
     unsigned cap = g->opts.trace_capacity ? g->opts.trace_capacity : 65536u;
@@ -213,14 +251,16 @@ sssp_status alloc_workspace(sssp_graph* g, Workspace& w, bool own_stream) {
     CK(cudaMalloc(&w.dist.p, n * 8), "allocating dist");
     w.dist.bytes = n * 8;
     CK(cudaMalloc(&w.expanded.p, (n + 31) / 32 * 4), "allocating the expansion bitmap");
-    CK(cudaMalloc(&w.bk.p, sizeof(BucketCtl) * kMaxBuckets), "allocating bucket counters");
-    CK(cudaMemset(w.bk.p, 0, sizeof(BucketCtl) * kMaxBuckets), "bucket counters");
+    CK(cudaMalloc(&w.bk.p, sizeof(BucketCtl) * (kMaxBuckets + 1)), "allocating bucket counters");
+    CK(cudaMemset(w.bk.p, 0, sizeof(BucketCtl) * (kMaxBuckets + 1)), "bucket counters");
     CK(cudaMalloc(&w.ctl.p, sizeof(Ctl)), "allocating control block");
     CK(cudaMemset(w.ctl.p, 0, sizeof(Ctl)), "control block");
     CK(cudaHostAlloc((void**)&w.h_ctl, sizeof(Ctl), cudaHostAllocDefault), "allocating pinned status block");
     std::memset(w.h_ctl, 0, sizeof(Ctl));
     for (auto& e : w.ev) CK(cudaEventCreate(&e), "creating events");
     if (own_stream) CK(cudaStreamCreateWithFlags(&w.own_stream, cudaStreamNonBlocking), "creating a slot stream");
+    sssp_status st = ensure_tasks(g, w, default_tcap(g));
+    if (st) return st;
     return ensure_ring(g, w, (g->opts.dist_bits == 64) ? 16 : 8, default_cap(g));
 }
 
@@ -294,6 +334,9 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
         cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
         p.keep_frac = want ? (float)std::min(1.0, (double)std::min(cur, use) / (double)want) : 0.0f;
     }
+    p.tasks = (SplitTask*)w.tasks.p;
+    p.tcap = w.tcap;
+    p.split_deg = split_degree(g, bt);
     p.k_max = k_max;
     p.timeout_ns = (unsigned long long)(g->opts.timeout_ms ? g->opts.timeout_ms : 60000u) * 1000000ull;
     return p;
@@ -337,7 +380,12 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     const unsigned k_max = kF ? 190u : (bits == 32 ? 31u : 63u);
     unsigned k = std::min(k0, k_max);
     const unsigned A0 = g->opts.active_init ? g->opts.active_init : 1u;
-    Head h0{0ull, pack_meta(0, k, A0, 0, 0)};
+    // initial floor of Delta (the controller never shrinks below it): the ring-span
+    // value w_max / B, below which one maximum-weight hop from the head already
+    // lands beyond the ring and is clipped ("the value of Delta should
+    // be large enough to minimize the chance of clipping"; reading R8)
+    const unsigned span = kF ? heuristic_k(g) : g->heur_k_span;
+    Head h0{0ull, pack_meta(0, k, A0, std::min(k, span), 0)};
     Params<DistT> p = make_params<DistT>(g, w, grid, bt, k_max, conc);
 
     const unsigned aux_grid = (unsigned)g->sm_count * 8 / conc + 1;
@@ -486,6 +534,7 @@ sssp_status settle_attempt(sssp_graph* g, Workspace& w, cudaStream_t s, int& bit
     }
     // aborted attempt: the ring holds leftovers -> clear it before anything else
     CK(cudaMemsetAsync(w.ring.p, 0xFF, w.ring.bytes, s), "clearing the bucket ring");
+    if (w.tasks.p) CK(cudaMemsetAsync(w.tasks.p, 0, w.tasks.bytes, s), "clearing the split-chunk queue");
     CK(cudaStreamSynchronize(s), "clearing the bucket ring");
     if (status & kStTimeout) return fail(SSSP_ERR_TIMEOUT, "device watchdog expired");
     if (status & kStBug) return fail(SSSP_ERR_CUDA, "internal invariant violated");
@@ -506,6 +555,8 @@ sssp_status settle_attempt(sssp_graph* g, Workspace& w, cudaStream_t s, int& bit
             return SSSP_OK;
         }
         const unsigned long long ncap = w.cap * 2;
+        sssp_status st3 = ensure_tasks(g, w, w.tcap * 2);
+        if (st3) return st3;
         w.ring.release();
         sssp_status st2 = ensure_ring(g, w, bits == 32 ? 8 : 16, ncap);
         if (st2) return st2;
@@ -669,7 +720,7 @@ void sssp_options_default(sssp_options* o) {
     o->util_lo_pct = 100;          // P:211 (reading R6)
     o->util_hi_pct = 400;
     o->waste_lo_permille = 450;    // reading R6: grow Delta only while < 45% of expansions are repeats
-    o->waste_hi_permille = 500;    //             shrink it while > 50% are (work <~ 2x Dijkstra)
+    o->waste_hi_permille = 600;    //             shrink it while > 60% are (work <~ 2.5x Dijkstra)
     o->period_us = 20;
     o->startup_permille = 20;
     o->dist_bits = 0;

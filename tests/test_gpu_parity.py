@@ -108,6 +108,10 @@ PERTURB = [
     dict(algorithm=sssp.SSSP_ALGO_NEAR_FAR), dict(algorithm=sssp.SSSP_ALGO_NEAR_FAR, delta_init=1),
     dict(algorithm=sssp.SSSP_ALGO_NEAR_FAR, delta_init=1 << 40), dict(algorithm=sssp.SSSP_ALGO_NEAR_FAR, ring_items=64),
     dict(algorithm=sssp.SSSP_ALGO_NEAR_FAR, grid_ctas=5), dict(flags=sssp.SSSP_FLAG_ADAPT_ACTIVE),
+    # hub splitting: 1-arc chunks (every multi-arc vertex splits; chunk-queue overflow + regrowth),
+    # small chunks on few CTAs, 64-bit distances, and splitting off
+    dict(split_degree=1), dict(split_degree=3, grid_ctas=3), dict(split_degree=2, dist_bits=64),
+    dict(split_degree=5, flags=sssp.SSSP_FLAG_NO_LOCAL), dict(split_degree=0xFFFFFFFF),
 ]
 
 
@@ -357,3 +361,26 @@ def test_float_rounding_fixture_and_errors():
     assert e.value.status == 1
     nz = sssp.Graph.from_csr(g, weights=np.array([-0.0, 1.0, 1.0], dtype=F32))   # -0.0 folds to +0.0
     assert nz.run(0).cpu().numpy().tolist() == [0.0, 0.0, 1.0]
+
+
+def test_hub_split_star():
+    """A source hub with 200K arcs (chunks of 1000 spread over the grid) plus a second-level hub,
+    zero weights and parallel arcs: bit-exact, and every arc of the hub counted exactly once."""
+    rng = np.random.default_rng(7)
+    n = 250_001
+    hub_arcs = 200_000
+    cols = [rng.integers(1, n, hub_arcs)]
+    ws = [rng.integers(0, 1000, hub_arcs)]
+    rows = [np.zeros(hub_arcs, np.int64)]
+    # vertex 1 is a second hub reached through the first
+    cols.append(rng.integers(0, n, 50_000)); ws.append(rng.integers(0, 5, 50_000)); rows.append(np.ones(50_000, np.int64))
+    src = np.concatenate(rows); dst = np.concatenate(cols); w = np.concatenate(ws)
+    order = np.lexsort((w, dst, src))
+    src, dst, w = src[order], dst[order], w[order]
+    off = np.zeros(n + 1, np.uint64)
+    np.add.at(off, src + 1, 1)
+    off = np.cumsum(off).astype(np.uint64)
+    g = gg.CSR(n, len(dst), off, dst.astype(np.uint32), w.astype(np.uint32))
+    for opt in (dict(), dict(split_degree=1000), dict(split_degree=1000, grid_ctas=2), dict(split_degree=0xFFFFFFFF)):
+        st = check(g, 0, **opt)
+        assert st["edges_relaxed"] >= st["reach_edges"]
