@@ -70,6 +70,10 @@ typedef enum sssp_status {
 #define SSSP_FLAG_NO_RETRY 0x4u  /* on worklist overflow return SSSP_ERR_WORKLIST_OVERFLOW instead of growing */
 #define SSSP_FLAG_NO_LOCAL 0x8u  /* publish every child through the ring (ablation of CTA-local continuation) */
 #define SSSP_FLAG_PROFILE 0x10u  /* accumulate per-phase SM-cycle counters (sssp_get_profile) */
+#define SSSP_FLAG_NO_WARP_LOCAL 0x80u /* ablation: no warp-local continuation (a warp running its own
+                                         head-bucket children hop after hop in the latency regime;
+                                         default on when the average degree is <= 8) */
+#define SSSP_FLAG_WARP_LOCAL 0x100u   /* force the warp-local continuation on whatever the degree */
 #define SSSP_FLAG_ADAPT_ACTIVE 0x40u  /* let the controller vary the number of active buckets;
                                         off by default: on our workloads it raised re-expansions */
 #define SSSP_FLAG_L2_PERSIST 0x20u /* reserve the L2 persisting set-aside for dist (raises the device-wide

@@ -69,6 +69,7 @@ struct Params {
     unsigned batch_min;
     unsigned share_shift;      // a CTA claims about avail >> share_shift items
     unsigned local_max;        // head-bucket children a CTA keeps for itself (0 = off)
+    unsigned warp_local;       // warp-local continuation in the latency regime (0 = off)
     unsigned max_backoff_ns;
     unsigned prof;             // SSSP_FLAG_PROFILE: accumulate per-phase cycles
     float keep_frac;           // fraction of dist covered by the L2 persisting set-aside
@@ -496,7 +497,11 @@ struct Smem {
     static constexpr size_t o_scan = o_rank + align16((size_t)kStage * 2);    // u32[BT]
     static constexpr size_t o_lv = o_scan + align16((size_t)BT * 4);          // u32[BT] kept children
     static constexpr size_t o_soff = o_lv + align16((size_t)BT * 4);          // u8[kStage]
-    static constexpr size_t bytes = o_soff + align16((size_t)kStage);
+    // warp-local continuation queues: kWQ {vertex, distance} per warp
+    static constexpr int kWQ = 128;
+    static constexpr size_t o_wqv = o_soff + align16((size_t)kStage);         // u32[BT/32 * kWQ]
+    static constexpr size_t o_wqd = o_wqv + align16((size_t)(BT / 32) * kWQ * 4);  // DistT[BT/32 * kWQ]
+    static constexpr size_t bytes = o_wqd + align16((size_t)(BT / 32) * kWQ * sizeof(DistT));
 };
 
 // --------------------------------------------------------------- kernel
@@ -522,6 +527,10 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     unsigned* s_scan = (unsigned*)(smem + L::o_scan);
     unsigned* s_lv = (unsigned*)(smem + L::o_lv);
     unsigned char* s_soff = (unsigned char*)(smem + L::o_soff);
+    constexpr unsigned kWQ = (unsigned)L::kWQ;
+    unsigned* s_wqv = (unsigned*)(smem + L::o_wqv);
+    DistT* s_wqd = (DistT*)(smem + L::o_wqd);
+    __shared__ unsigned s_wst[5];  // warp-local continuation: expanded, first, edges, stale, kept
 
     __shared__ unsigned s_cnt[kMaxBuckets];
     __shared__ unsigned long long s_base[kMaxBuckets];
@@ -542,6 +551,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
 
     if (tid < (int)kMaxBuckets) s_cnt[tid] = 0;
     if (tid < (int)kProfCounters) s_prof[tid] = 0;
+    if (tid < 5) s_wst[tid] = 0;
     if (tid == 0) {
         s_total = 0;
         s_lnext = 0;
@@ -614,6 +624,9 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         // work): with plentiful work it starves the other CTAs of head-bucket items
         // (measured: RMAT 2x slower with a full-CTA cap)
         const unsigned lcap = got * 2 <= (unsigned)BT ? local_max : 0u;
+        // warp-local continuation (same regime): a warp runs its own head-bucket
+        // children hop after hop with no CTA barrier (D9)
+        const bool wlc = lcap != 0 && p.warp_local != 0;
 
         // ------------------------------------------------------------ pop + stale check
         const Head hd = s_head;
@@ -758,6 +771,104 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                                   : make_uint2(0u, 0u);
                 }
             };
+            // head-bucket children stay on chip: first in this warp's own queue (warp-local
+            // continuation), then in the CTA's next batch (warp-aggregated slot grabs)
+            unsigned wq_n = 0;  // warp-uniform fill of this warp's queue
+            const unsigned wq0 = (unsigned)warp * kWQ;
+            auto keep = [&](const bool want, const unsigned v, const unsigned long long ndv) -> bool {
+                bool kept = false;
+                if (wlc) {
+                    const unsigned wm = __ballot_sync(FULL, want);
+                    if (wm) {
+                        const unsigned pos = wq_n + __popc(wm & lt_mask);
+                        if (want && pos < kWQ) {
+                            s_wqv[wq0 + pos] = v;
+                            s_wqd[wq0 + pos] = (DistT)ndv;
+                            kept = true;
+                        }
+                        const unsigned nn = wq_n + __popc(wm);
+                        if (lane == 0) atomicAdd(&s_wst[4], (nn < kWQ ? nn : kWQ) - wq_n);
+                        wq_n = nn < kWQ ? nn : kWQ;
+                    }
+                }
+                if (lcap) {
+                    const bool w2 = want && !kept;
+                    const unsigned lm = __ballot_sync(FULL, w2);
+                    if (lm) {
+                        const int leader = __ffs(lm) - 1;
+                        unsigned pos = 0;
+                        if (lane == leader) pos = atomicAdd(&s_lnext, (unsigned)__popc(lm));
+                        pos = __shfl_sync(FULL, pos, leader) + __popc(lm & lt_mask);
+                        if (w2 && pos < lcap) {
+                            s_lv[pos] = v;
+                            s_ld[pos] = (DistT)ndv;
+                            kept = true;
+                        }
+                    }
+                }
+                return kept;
+            };
+            // everything else: warp-aggregated staging for the CTA flush at batch end
+            // (or direct publication when the staging area is full)
+            auto emit = [&](const bool pg, const unsigned v, const unsigned long long ndv, const unsigned o) {
+                const unsigned act = __ballot_sync(FULL, pg);
+                if (!act) return;
+                // warp-aggregated staging slot for the CTA flush at batch end
+                const int leader = __ffs(act) - 1;
+                const unsigned nact = (unsigned)__popc(act);
+                unsigned pos = 0;
+                if (lane == leader) pos = atomicAdd(&s_total, nact);
+                pos = __shfl_sync(FULL, pos, leader);
+                if (pos + nact <= (unsigned)kStage) {
+                    if (pg) {
+                        const unsigned peers = __match_any_sync(act, o);
+                        const int pl = __ffs(peers) - 1;
+                        unsigned r0 = 0;
+                        if (lane == pl) r0 = atomicAdd(&s_cnt[o], (unsigned)__popc(peers));
+                        r0 = __shfl_sync(peers, r0, pl) + __popc(peers & lt_mask);
+                        const unsigned my = pos + __popc(act & lt_mask);
+                        s_items[my] = IT::make(v, ndv);
+                        s_soff[my] = (unsigned char)o;
+                        s_rank[my] = (unsigned short)r0;
+                    }
+                } else {
+                    // staging full (hubs): mark the slots this warp took as holes and
+                    // publish directly -- one reserve/avail pair per (warp, bucket)
+                    if (pg) {
+                        const unsigned my = pos + __popc(act & lt_mask);
+                        if (my < (unsigned)kStage) s_soff[my] = 0xFF;
+                        const unsigned peers = __match_any_sync(act, o);
+                        const int pl = __ffs(peers) - 1;
+                        const unsigned sl = (hs + o) & nbm;
+                        unsigned long long b0 = 0;
+                        if (lane == pl) {
+                            const unsigned c = (unsigned)__popc(peers);
+                            b0 = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
+                            if (b0 + c > p.cap) {
+                                const unsigned long long cl = ld_relaxed_u64(&p.bk[sl].claim.v);
+                                if (b0 + c - p.cap > cl) atomicOr(&p.ctl->status, kStRingOverflow);
+                            }
+                            atomicAdd(&s_direct, c);
+                        }
+                        b0 = __shfl_sync(peers, b0, pl);
+                        const unsigned long long idx = b0 + __popc(peers & lt_mask);
+                        char* sp = p.ring + ((size_t)sl * p.cap + (idx & (p.cap - 1))) * IT::kBytes;
+                        bool ok = true;
+                        if (idx >= p.cap) {
+                            unsigned spins = 0;
+                            while (!IT::empty(sp)) {
+                                if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) {
+                                    ok = false;
+                                    break;
+                                }
+                            }
+                        }
+                        if (ok) IT::store(sp, IT::make(v, ndv));
+                        __syncwarp(peers);
+                        if (lane == pl) atomicAdd(&p.bk[sl].avail.v, (unsigned long long)__popc(peers));
+                    }
+                }
+            };
             // relax + push of one round whose arcs are loaded
             auto body = [&](const unsigned base, const unsigned (&own)[EPT], const uint2 (&a)[EPT]) {
                 unsigned long long nd[EPT];
@@ -794,80 +905,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 for (int j = 0; j < EPT; ++j) {
                     if (!__any_sync(FULL, push[j])) continue;
                     const unsigned o = push[j] ? bucket_of<kF>(nd[j], k, hd.h, p.nb) : 0u;
-                    // head-bucket children stay in this CTA (warp-aggregated slot grab)
-                    bool kept = false;
-                    if (lcap) {
-                        const unsigned lm = __ballot_sync(FULL, push[j] && o == 0);
-                        if (lm) {
-                            const int leader = __ffs(lm) - 1;
-                            unsigned pos = 0;
-                            if (lane == leader) pos = atomicAdd(&s_lnext, (unsigned)__popc(lm));
-                            pos = __shfl_sync(FULL, pos, leader) + __popc(lm & lt_mask);
-                            if (push[j] && o == 0 && pos < lcap) {
-                                s_lv[pos] = a[j].x;
-                                s_ld[pos] = (DistT)nd[j];
-                                kept = true;
-                            }
-                        }
-                    }
-                    const bool pg = push[j] && !kept;
-                    const unsigned act = __ballot_sync(FULL, pg);
-                    if (!act) continue;
-                    // warp-aggregated staging slot for the CTA flush at batch end
-                    const int leader = __ffs(act) - 1;
-                    const unsigned nact = (unsigned)__popc(act);
-                    unsigned pos = 0;
-                    if (lane == leader) pos = atomicAdd(&s_total, nact);
-                    pos = __shfl_sync(FULL, pos, leader);
-                    if (pos + nact <= (unsigned)kStage) {
-                        if (pg) {
-                            const unsigned peers = __match_any_sync(act, o);
-                            const int pl = __ffs(peers) - 1;
-                            unsigned r0 = 0;
-                            if (lane == pl) r0 = atomicAdd(&s_cnt[o], (unsigned)__popc(peers));
-                            r0 = __shfl_sync(peers, r0, pl) + __popc(peers & lt_mask);
-                            const unsigned my = pos + __popc(act & lt_mask);
-                            s_items[my] = IT::make(a[j].x, nd[j]);
-                            s_soff[my] = (unsigned char)o;
-                            s_rank[my] = (unsigned short)r0;
-                        }
-                    } else {
-                        // staging full (hubs): mark the slots this warp took as holes and
-                        // publish directly -- one reserve/avail pair per (warp, bucket)
-                        if (pg) {
-                            const unsigned my = pos + __popc(act & lt_mask);
-                            if (my < (unsigned)kStage) s_soff[my] = 0xFF;
-                            const unsigned peers = __match_any_sync(act, o);
-                            const int pl = __ffs(peers) - 1;
-                            const unsigned sl = (hs + o) & nbm;
-                            unsigned long long b0 = 0;
-                            if (lane == pl) {
-                                const unsigned c = (unsigned)__popc(peers);
-                                b0 = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
-                                if (b0 + c > p.cap) {
-                                    const unsigned long long cl = ld_relaxed_u64(&p.bk[sl].claim.v);
-                                    if (b0 + c - p.cap > cl) atomicOr(&p.ctl->status, kStRingOverflow);
-                                }
-                                atomicAdd(&s_direct, c);
-                            }
-                            b0 = __shfl_sync(peers, b0, pl);
-                            const unsigned long long idx = b0 + __popc(peers & lt_mask);
-                            char* sp = p.ring + ((size_t)sl * p.cap + (idx & (p.cap - 1))) * IT::kBytes;
-                            bool ok = true;
-                            if (idx >= p.cap) {
-                                unsigned spins = 0;
-                                while (!IT::empty(sp)) {
-                                    if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) {
-                                        ok = false;
-                                        break;
-                                    }
-                                }
-                            }
-                            if (ok) IT::store(sp, IT::make(a[j].x, nd[j]));
-                            __syncwarp(peers);
-                            if (lane == pl) atomicAdd(&p.bk[sl].avail.v, (unsigned long long)__popc(peers));
-                        }
-                    }
+                    const bool kept = keep(push[j] && o == 0, a[j].x, nd[j]);
+                    emit(push[j] && !kept, a[j].x, nd[j], o);
                 }
             };
             if (PIPE && we > wb + 32 * EPT) {
@@ -893,6 +932,89 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     uint2 a[EPT];
                     fetch(base, own, a);
                     body(base, own, a);
+                }
+            }
+            // ------------------------------------------------ warp-local continuation
+            // Latency regime only (road-like graphs: a few hundred items per bucket,
+            // thousands of dependent hops).  The warp pops up to 32 of its own kept
+            // children (one per lane, LIFO), re-checks staleness while loading the row,
+            // relaxes each child's arcs EPT at a time with no filter load, and keeps /
+            // emits the improved ones exactly like the batch does -- one hop costs three
+            // dependent L2 round trips (row, arcs, atomicMin) and no CTA barrier.  The
+            // children are covered by this batch's own pending count (the batch
+            // completes after its warps' queues drain), so no counter is touched.
+            // Rows longer than kWDeg go back through the ring (head bucket).
+            constexpr unsigned kWDeg = 8u * EPT;
+            while (wq_n > 0) {
+                const unsigned take = wq_n < 32u ? wq_n : 32u;
+                const unsigned st0 = wq_n - take;
+                const bool has = lane < (int)take;
+                unsigned v = 0;
+                unsigned long long dv = kInf;
+                if (has) {
+                    v = s_wqv[wq0 + st0 + lane];
+                    dv = (unsigned long long)s_wqd[wq0 + st0 + lane];
+                }
+                __syncwarp();
+                wq_n = st0;
+                unsigned long long b = 0, e = 0;
+                bool lv = false;
+                if (has) {
+                    const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
+                    b = ld_stream_u64(p.off + v, pol_stream);
+                    e = ld_stream_u64(p.off + v + 1, pol_stream);
+                    lv = cur >= dv;
+                }
+                const bool big = lv && (e - b) > kWDeg;
+                emit(big, v, dv, 0u);  // long rows: back to the head bucket through the ring
+                lv = lv && !big;
+                bool fst = false;
+                if (lv && p.dynamic) {
+                    const unsigned bit = 1u << (v & 31);
+                    fst = (atomicOr(p.expanded + (v >> 5), bit) & bit) == 0;
+                }
+                const unsigned deg = lv ? (unsigned)(e - b) : 0u;
+                const unsigned nl = (unsigned)__popc(__ballot_sync(FULL, lv));
+                const unsigned nf = (unsigned)__popc(__ballot_sync(FULL, fst));
+                const unsigned ns = (unsigned)__popc(__ballot_sync(FULL, has && !lv && !big));
+                const unsigned sumdeg = __reduce_add_sync(FULL, deg);
+                const unsigned maxdeg = __reduce_max_sync(FULL, deg);
+                if (lane == 0) {
+                    if (nl) atomicAdd(&s_wst[0], nl);
+                    if (nf) atomicAdd(&s_wst[1], nf);
+                    if (sumdeg) atomicAdd(&s_wst[2], sumdeg);
+                    if (ns) atomicAdd(&s_wst[3], ns);
+                }
+                for (unsigned kk = 0; kk < maxdeg; kk += EPT) {
+                    uint2 a[EPT];
+                    unsigned long long nd[EPT];
+                    DistT old[EPT];
+                    bool push[EPT];
+#pragma unroll
+                    for (int j = 0; j < EPT; ++j)
+                        a[j] = kk + j < deg ? ld_stream_u2(p.adj + b + kk + j, pol_stream) : make_uint2(0u, 0u);
+#pragma unroll
+                    for (int j = 0; j < EPT; ++j) {
+                        push[j] = false;
+                        old[j] = (DistT)0;
+                        nd[j] = kk + j < deg ? relax_sum<kF>(dv, a[j].y) : kInf;
+                        if (kk + j < deg) {
+                            if (sum_unusable<kF>(nd[j], kInf)) {
+                                if (!kF) atomicOr(&p.ctl->status, kStDistOverflow);
+                            } else {
+                                old[j] = atomic_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
+                                push[j] = true;
+                            }
+                        }
+                    }
+#pragma unroll
+                    for (int j = 0; j < EPT; ++j) {
+                        push[j] = push[j] && nd[j] < (unsigned long long)old[j];
+                        if (!__any_sync(FULL, push[j])) continue;
+                        const unsigned o = push[j] ? bucket_of<kF>(nd[j], k, hd.h, p.nb) : 0u;
+                        const bool kept = keep(push[j] && o == 0, a[j].x, nd[j]);
+                        emit(push[j] && !kept, a[j].x, nd[j], o);
+                    }
                 }
             }
         }
@@ -972,7 +1094,16 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         // ------------------------------------------------------------ complete
         __syncthreads();  // s_lnext final (also covers the E == 0 case)
         const unsigned kept = s_lnext < lcap ? s_lnext : lcap;
+        const unsigned w_exp = s_wst[0], w_first = s_wst[1], w_kept = s_wst[4];
         if (tid == 0) {
+            if (wlc) {
+                c_vert += w_exp;
+                c_edges += s_wst[2];
+                c_stale += s_wst[3];
+                c_push += s_wst[4];
+                c_local += s_wst[4];
+                s_wst[0] = s_wst[1] = s_wst[2] = s_wst[3] = s_wst[4] = 0;
+            }
             // one atomic: the kept children inherit the parents' accounting
             if (got > kept) atomicAdd(&p.bk[slot].done.v, (unsigned long long)(got - kept));
             else if (kept > got) atomicAdd(&p.bk[slot].local.v, (unsigned long long)(kept - got));
@@ -983,11 +1114,11 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         if (p.dynamic && warp == 0) {
             unsigned run_ctl = 0;
             if (lane == 0) {
-                if (nexp) {
-                    atomicAdd(&p.ctl->g_exp, (unsigned long long)nexp);
-                    atomicAdd(&p.ctl->g_first, (unsigned long long)nfirst);
+                if (nexp + w_exp) {
+                    atomicAdd(&p.ctl->g_exp, (unsigned long long)(nexp + w_exp));
+                    atomicAdd(&p.ctl->g_first, (unsigned long long)(nfirst + w_first));
                 }
-                if (kept) atomicAdd(&p.ctl->g_push, (unsigned long long)kept);
+                if (kept + w_kept) atomicAdd(&p.ctl->g_push, (unsigned long long)(kept + w_kept));
                 const unsigned long long now = globaltimer();
                 const unsigned long long last = ld_relaxed_u64(&p.ctl->last_ctl_ns);
                 if (now - last > p.period_ns && atomicCAS(&p.ctl->last_ctl_ns, last, now) == last) run_ctl = 1;

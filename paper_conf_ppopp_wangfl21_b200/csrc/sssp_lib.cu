@@ -170,9 +170,9 @@ template <typename DistT, int BT, bool kF = false, int EPT = 4, int MINB = 1024 
 KVariant kvar() {
     return KVariant{(void*)adds_persistent_kernel<DistT, BT, EPT, MINB, PIPE, kF>, Smem<DistT, BT, EPT>::bytes};
 }
-// SSSP_KVAR (experiments): 0 default; 1 pipelined 512x2/SM EPT 4; 2 pipelined 512x1/SM EPT 8;
+// SSSP_KVAR (experiments): 0 default (= 1 for 32-bit 512-thread CTAs); 1 pipelined 512x2/SM EPT 4; 2 pipelined 512x1/SM EPT 8;
 // 3 pipelined 1024x1/SM EPT 4; 4 pipelined 512x1/SM EPT 4; 5 plain 512x1/SM EPT 8;
-// 6 pipelined 256x2/SM EPT 8
+// 6 pipelined 256x2/SM EPT 8; 7 plain 512x2/SM EPT 4 (the pre-pipeline default)
 static int kvar_env() {
     const char* e = std::getenv("SSSP_KVAR");
     return e ? std::atoi(e) : 0;
@@ -188,7 +188,8 @@ KVariant persistent_variant(int bits, int bt, bool f32) {
         if (kv == 5) return kvar<uint32_t, 512, false, 8, 1, false>();
         if (kv == 6) return kvar<uint32_t, 256, false, 8, 2, true>();
         if (bt == 128) return kvar<uint32_t, 128>();
-        if (bt == 512) return kvar<uint32_t, 512>();
+        if (kv == 7) return kvar<uint32_t, 512>();  // 512 x 2/SM without the software pipeline (A/B)
+        if (bt == 512) return kvar<uint32_t, 512, false, 4, 2, true>();  // default: pipelined
         if (bt == 1024) return kvar<uint32_t, 1024>();
         return kvar<uint32_t, 256>();
     }
@@ -308,6 +309,11 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
     while ((1u << (sh + 1)) <= grid) ++sh;  // floor(log2 grid)
     p.share_shift = sh > 2 ? sh - 2 : 0;
     p.local_max = (g->opts.flags & SSSP_FLAG_NO_LOCAL) ? 0u : (g->opts.local_max ? g->opts.local_max : 128u);
+    // warp-local continuation pays on low-degree graphs (road-like: each lane's row fits
+    // one or two rounds of EPT arcs); on ER (degree 32) it serialised what the ring spreads
+    // over CTAs (measured +13 %), so it is on by default only for average degree <= 8
+    p.warp_local = (g->opts.flags & (SSSP_FLAG_NO_LOCAL | SSSP_FLAG_NO_WARP_LOCAL)) ? 0u
+                   : (g->opts.flags & SSSP_FLAG_WARP_LOCAL) || g->m <= 8ull * g->n ? 1u : 0u;
     p.max_backoff_ns = g->opts.max_backoff_ns ? g->opts.max_backoff_ns : 2048u;
     p.prof = (g->opts.flags & SSSP_FLAG_PROFILE) ? 1u : 0u;
     p.expanded = (unsigned*)w.expanded.p;

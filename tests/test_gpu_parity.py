@@ -112,6 +112,8 @@ PERTURB = [
     # small chunks on few CTAs, 64-bit distances, and splitting off
     dict(split_degree=1), dict(split_degree=3, grid_ctas=3), dict(split_degree=2, dist_bits=64),
     dict(split_degree=5, flags=sssp.SSSP_FLAG_NO_LOCAL), dict(split_degree=0xFFFFFFFF),
+    # warp-local continuation off / with a 1-item CTA-level cap; 1024-thread CTAs
+    dict(flags=sssp.SSSP_FLAG_NO_WARP_LOCAL), dict(flags=sssp.SSSP_FLAG_WARP_LOCAL, local_max=1, grid_ctas=2), dict(block_threads=1024),
 ]
 
 
