@@ -277,6 +277,25 @@ def run_ours(args, world, rank, local):
                "h2d_bytes_per_step": int(g.row_offsets.nbytes + g.col.nbytes + g.w.nbytes),
                "d2h_bytes_per_step": int(8 * g.n), "steps": k_e,
                "path": "sssp_graph_create(pinned host CSR) + sssp_run(host dist_out) + destroy"}
+        # serving shape: the graph stays resident (uploaded once, like model weights), every
+        # query is a source in and a full distance vector out to pinned host memory
+        barrier()
+        t0 = time.perf_counter()
+        Er = 0
+        for i in range(args.steps):
+            sssp._check(sssp.lib().sssp_run(G._h, int(srcs[args.warmup + i]), dist_h.data_ptr(),
+                                            sssp._stream_ptr(stream)))
+            Er += G.stats()["reach_edges"]
+        torch.cuda.synchronize(dev)
+        tr = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
+        er = torch.tensor([float(Er)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(tr, op=dist.ReduceOp.MAX)
+            dist.all_reduce(er, op=dist.ReduceOp.SUM)
+        e2e["resident_graph"] = {"value": er.item() / tr.item() / 1e9, "unit": "GTEPS", "steps": args.steps,
+                                 "h2d_bytes_per_step": 0, "d2h_bytes_per_step": int(8 * g.n),
+                                 "path": "sssp_run(resident graph, host dist_out): source in, distances "
+                                         "copied to pinned host memory inside the call"}
 
     if rank == 0:
         hbm, peak_kind = peaks()

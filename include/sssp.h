@@ -74,6 +74,9 @@ typedef enum sssp_status {
                                          head-bucket children hop after hop in the latency regime;
                                          default on when the average degree is <= 8) */
 #define SSSP_FLAG_WARP_LOCAL 0x100u   /* force the warp-local continuation on whatever the degree */
+#define SSSP_FLAG_FILTER16 0x200u     /* experiment (off by default, measured slower): filter relaxations
+                                         with a 16-bit upper-bound array of dist (half its L2 footprint)
+                                         instead of a load of dist itself; D11 */
 #define SSSP_FLAG_ADAPT_ACTIVE 0x40u  /* let the controller vary the number of active buckets;
                                         off by default: on our workloads it raised re-expansions */
 #define SSSP_FLAG_L2_PERSIST 0x20u /* reserve the L2 persisting set-aside for dist (raises the device-wide

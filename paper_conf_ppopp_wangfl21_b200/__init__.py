@@ -36,6 +36,7 @@ SSSP_FLAG_L2_PERSIST = 0x20
 SSSP_FLAG_ADAPT_ACTIVE = 0x40
 SSSP_FLAG_NO_WARP_LOCAL = 0x80
 SSSP_FLAG_WARP_LOCAL = 0x100
+SSSP_FLAG_FILTER16 = 0x200
 PROFILE_FIELDS = ["cyc_claim", "cyc_idle", "cyc_pop", "cyc_scan", "cyc_rounds", "cyc_flush", "cyc_complete",
                   "cyc_total", "n_ring_batches", "n_local_batches", "n_idle", "n_flush", "n_rounds", "n_ctas",
                   "cyc_window", "n_windows"]

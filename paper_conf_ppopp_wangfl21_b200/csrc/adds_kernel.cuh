@@ -70,6 +70,9 @@ struct Params {
     unsigned share_shift;      // a CTA claims about avail >> share_shift items
     unsigned local_max;        // head-bucket children a CTA keeps for itself (0 = off)
     unsigned warp_local;       // warp-local continuation in the latency regime (0 = off)
+    unsigned exp;              // experiment toggles (SSSP_EXP env, A/B on one box; 0 = production)
+    unsigned short* filt;      // n x u16 upper bounds of dist in units of 2^filt_shift (nullptr = off)
+    unsigned filt_shift;
     unsigned max_backoff_ns;
     unsigned prof;             // SSSP_FLAG_PROFILE: accumulate per-phase cycles
     float keep_frac;           // fraction of dist covered by the L2 persisting set-aside
@@ -359,6 +362,21 @@ __device__ __forceinline__ unsigned bucket_of(unsigned long long nd, unsigned k,
     }
 }
 
+// --------------------------------------------------------------- 16-bit filter (D11)
+// filt[v] = ceil(x / 2^s) for some value x that dist[v] held at some time (so, since
+// dist only decreases, filt[v] << s >= dist[v] forever), 0xFFFF = no bound.  The
+// relaxation filter reads this 2-byte array (half the L2 footprint of dist) instead
+// of dist: nd >= filt[v] << s  =>  nd >= dist[v]  =>  the arc cannot improve.  Any
+// racing plain store keeps the invariant, because every value ever written is a
+// bound of the (monotone) distance.
+__device__ __forceinline__ unsigned long long filt_bound(unsigned short f, unsigned s) {
+    return f == 0xFFFFu ? ~0ull : ((unsigned long long)f << s);
+}
+__device__ __forceinline__ unsigned short filt_enc(unsigned long long x, unsigned s) {
+    const unsigned long long q = (x + ((1ull << s) - 1)) >> s;
+    return q >= 0xFFFFull ? (unsigned short)0xFFFFu : (unsigned short)q;
+}
+
 // --------------------------------------------------------------- claim (A4)
 // Warp-cooperative: status + head (lane 0), then the A active buckets' avail
 // gates (idle CTAs poll here, so every extra line read lands on a hot L2 slice);
@@ -632,7 +650,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         const Head hd = s_head;
         const unsigned hs = meta_hs(hd.meta), k = meta_k(hd.meta);
         unsigned deg = 0;
-        bool live = false, first = false;
+        bool live = false;
+        unsigned fword = 0, fbit = 0;  // expansion-bitmap word before our atomicOr (consumed at batch end)
         if (is_task) {
             // a hub-split chunk: one vertex, len arcs, charged to the slot it carries
             if (tid == 0) {
@@ -683,7 +702,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     live = true;
                     if (p.dynamic) {  // work-waste signal: is this v's first expansion?
                         const unsigned bit = 1u << (v & 31);
-                        first = (atomicOr(p.expanded + (v >> 5), bit) & bit) == 0;
+                        fword = atomicOr(p.expanded + (v >> 5), bit);  // result not waited for until the batch ends
+                        fbit = bit;
                     }
                     if (p.split_deg && deg > p.split_deg) deg = spawn_chunks(p, v, d, b, deg, slot);
                 }
@@ -705,7 +725,6 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         }
         if (lane == 31) s_wsum[warp] = x;
         const int nlive = __syncthreads_count(live);
-        const int nfirst = p.dynamic ? __syncthreads_count(first) : 0;
         if (warp == 0) {
             const unsigned ws = lane < kWarps ? s_wsum[lane] : 0;
             unsigned inc = ws;
@@ -784,6 +803,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         if (want && pos < kWQ) {
                             s_wqv[wq0 + pos] = v;
                             s_wqd[wq0 + pos] = (DistT)ndv;
+                            if (!(p.exp & 1u)) prefetch_l1(p.off + v);  // the next hop reads this row from L1
                             kept = true;
                         }
                         const unsigned nn = wq_n + __popc(wm);
@@ -881,8 +901,11 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
 #pragma unroll
                 for (int j = 0; j < EPT; ++j)  // EPT independent L2 gathers in flight
-                    cur[j] = (nd[j] < kInf && !tiny) ? ld_keep(p.dist + a[j].x, pol_keep)
-                                                     : (nd[j] < kInf ? DistInf<DistT>::value : (DistT)0);
+                    cur[j] = (nd[j] < kInf && !tiny)
+                                 ? (p.filt ? (DistT)min(filt_bound(ld_filt(p.filt + a[j].x), p.filt_shift),
+                                                        (unsigned long long)DistInf<DistT>::value)
+                                           : ld_keep(p.dist + a[j].x, pol_keep))
+                                 : (nd[j] < kInf ? DistInf<DistT>::value : (DistT)0);
                 DistT old[EPT];
                 bool tried[EPT];
 #pragma unroll
@@ -900,7 +923,10 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     }
                 }
 #pragma unroll
-                for (int j = 0; j < EPT; ++j) push[j] = tried[j] && nd[j] < (unsigned long long)old[j];
+                for (int j = 0; j < EPT; ++j) {
+                    push[j] = tried[j] && nd[j] < (unsigned long long)old[j];
+                    if (push[j] && p.filt) st_filt(p.filt + a[j].x, filt_enc(nd[j], p.filt_shift));
+                }
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {
                     if (!__any_sync(FULL, push[j])) continue;
@@ -957,13 +983,21 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
                 __syncwarp();
                 wq_n = st0;
+                // no stale re-check: the child was improved by this warp a hop ago (a
+                // superseded child only costs a redundant relaxation), so the hop waits on
+                // the L1-prefetched row alone
                 unsigned long long b = 0, e = 0;
-                bool lv = false;
+                bool lv = has;
                 if (has) {
-                    const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
-                    b = ld_stream_u64(p.off + v, pol_stream);
-                    e = ld_stream_u64(p.off + v + 1, pol_stream);
-                    lv = cur >= dv;
+                    if (p.exp & 1u) {  // A/B: previous hop shape (stale re-check, L2 row loads)
+                        const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
+                        b = ld_stream_u64(p.off + v, pol_stream);
+                        e = ld_stream_u64(p.off + v + 1, pol_stream);
+                        lv = cur >= dv;
+                    } else {
+                        b = ld_ca_u64(p.off + v);
+                        e = ld_ca_u64(p.off + v + 1);
+                    }
                 }
                 const bool big = lv && (e - b) > kWDeg;
                 emit(big, v, dv, 0u);  // long rows: back to the head bucket through the ring
@@ -1010,6 +1044,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
 #pragma unroll
                     for (int j = 0; j < EPT; ++j) {
                         push[j] = push[j] && nd[j] < (unsigned long long)old[j];
+                        if (push[j] && p.filt) st_filt(p.filt + a[j].x, filt_enc(nd[j], p.filt_shift));
                         if (!__any_sync(FULL, push[j])) continue;
                         const unsigned o = push[j] ? bucket_of<kF>(nd[j], k, hd.h, p.nb) : 0u;
                         const bool kept = keep(push[j] && o == 0, a[j].x, nd[j]);
@@ -1092,7 +1127,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         }
 
         // ------------------------------------------------------------ complete
-        __syncthreads();  // s_lnext final (also covers the E == 0 case)
+        // s_lnext final (also covers the E == 0 case); first expansions for the controller
+        const int nfirst = __syncthreads_count(fbit != 0 && (fword & fbit) == 0);
         const unsigned kept = s_lnext < lcap ? s_lnext : lcap;
         const unsigned w_exp = s_wst[0], w_first = s_wst[1], w_kept = s_wst[4];
         if (tid == 0) {

@@ -42,11 +42,15 @@ __global__ void interleave_kernel(const unsigned* __restrict__ col, const unsign
 
 template <typename DistT>
 __global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned source, Ctl* ctl, BucketCtl* bk,
-                                char* ring, unsigned long long cap, Head h0, unsigned* expanded) {
+                                char* ring, unsigned long long cap, Head h0, unsigned* expanded,
+                                unsigned short* filt) {
     using IT = ItemT<DistT>;
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
     for (unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
         dist[v] = (v == source) ? (DistT)0 : DistInf<DistT>::value;
+    if (filt)
+        for (unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+            filt[v] = (v == source) ? (unsigned short)0 : (unsigned short)0xFFFFu;
     const unsigned long long nw = ((unsigned long long)n + 31) / 32;
     for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += stride)
         expanded[i] = 0u;

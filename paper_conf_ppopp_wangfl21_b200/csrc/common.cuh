@@ -202,6 +202,15 @@ __device__ __forceinline__ unsigned long long ld_keep(const unsigned long long* 
     asm volatile("ld.global.cg.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(r) : "l"(a), "l"(pol));
     return r;
 }
+// 16-bit upper-bound filter of dist (D11)
+__device__ __forceinline__ unsigned short ld_filt(const unsigned short* a) {
+    unsigned short r;
+    asm volatile("ld.global.cg.u16 %0, [%1];" : "=h"(r) : "l"(a));
+    return r;
+}
+__device__ __forceinline__ void st_filt(unsigned short* a, unsigned short v) {
+    asm volatile("st.global.cg.u16 [%0], %1;" ::"l"(a), "h"(v) : "memory");
+}
 __device__ __forceinline__ unsigned atomic_min_keep(unsigned* a, unsigned v, unsigned long long pol) {
     unsigned r;
     asm volatile("atom.global.L2::cache_hint.min.u32 %0, [%1], %2, %3;" : "=r"(r) : "l"(a), "r"(v), "l"(pol) : "memory");
@@ -252,6 +261,13 @@ __device__ __forceinline__ void cp_async_8(unsigned sdst, const void* gsrc, unsi
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
+// non-blocking L1 prefetch of a read-only line (row offsets of a child kept for the next hop)
+__device__ __forceinline__ void prefetch_l1(const void* p) { asm volatile("prefetch.global.L1 [%0];" ::"l"(p)); }
+__device__ __forceinline__ unsigned long long ld_ca_u64(const unsigned long long* a) {
+    unsigned long long r;
+    asm volatile("ld.global.ca.u64 %0, [%1];" : "=l"(r) : "l"(a));
+    return r;
+}
 // non-blocking L2 prefetch (no register result, nothing waits on it)
 __device__ __forceinline__ void prefetch_l2(const void* p) {
     asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(p));

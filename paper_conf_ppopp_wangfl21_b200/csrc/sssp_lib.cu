@@ -73,6 +73,7 @@ struct Workspace {
     DevBuf ring;        // nb * cap * item bytes
     DevBuf bk, ctl, trace, expanded;
     DevBuf tasks;                   // hub-split chunk queue (SplitTask[tcap])
+    DevBuf filt;                    // n x u16 upper-bound filter of dist (D11)
     unsigned long long tcap = 0;
     unsigned long long cap = 0;
     int ring_item_bytes = 0;
@@ -92,6 +93,7 @@ struct Workspace {
         trace.release();
         expanded.release();
         tasks.release();
+        filt.release();
         nf_piles.release();
         nf_cnt.release();
         if (h_ctl) cudaFreeHost(h_ctl);
@@ -121,6 +123,7 @@ struct sssp_graph {
     DevBuf scratch, hostout;
     cudaEvent_t bev[2] = {nullptr, nullptr};  // batch start / end on the caller's stream
     int cur_bits = 32;       // 64 after a 32-bit overflow was observed (sticky)
+    unsigned filt_shift_hint = 0;  // 1 + filter resolution fitted to the last run's max distance
     size_t persist_max = 0;  // device's L2 persisting set-aside limit (bytes)
     bool busy = false;
     bool async_pending = false;
@@ -252,6 +255,7 @@ sssp_status alloc_workspace(sssp_graph* g, Workspace& w, bool own_stream) {
     CK(cudaMalloc(&w.dist.p, n * 8), "allocating dist");
     w.dist.bytes = n * 8;
     CK(cudaMalloc(&w.expanded.p, (n + 31) / 32 * 4), "allocating the expansion bitmap");
+    CK(cudaMalloc(&w.filt.p, n * 2 + 16), "allocating the 16-bit filter");
     CK(cudaMalloc(&w.bk.p, sizeof(BucketCtl) * (kMaxBuckets + 1)), "allocating bucket counters");
     CK(cudaMemset(w.bk.p, 0, sizeof(BucketCtl) * (kMaxBuckets + 1)), "bucket counters");
     CK(cudaMalloc(&w.ctl.p, sizeof(Ctl)), "allocating control block");
@@ -340,6 +344,21 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
         cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
         p.keep_frac = want ? (float)std::min(1.0, (double)std::min(cur, use) / (double)want) : 0.0f;
     }
+    // 16-bit filter (D11, opt-in): integer weights only (distances beyond
+    // 65534 * 2^s simply have no bound and go to the atomic)
+    {
+        const bool on = !g->f32 && (g->opts.flags & SSSP_FLAG_FILTER16);
+        unsigned lg = 0;
+        while (lg < 31 && (2u << lg) <= g->max_w) ++lg;  // floor(log2 max_w)
+        p.filt = on ? (unsigned short*)w.filt.p : nullptr;
+        // first run on a graph: 2^s = max_w / 16; afterwards the resolution that maps the
+        // previous run's largest distance below 60000 (the result never depends on it)
+        p.filt_shift = g->filt_shift_hint ? g->filt_shift_hint - 1 : (lg > 4 ? lg - 4 : 0);
+    }
+    {
+        const char* e = std::getenv("SSSP_EXP");
+        p.exp = e ? (unsigned)std::strtoul(e, nullptr, 0) : 0u;
+    }
     p.tasks = (SplitTask*)w.tasks.p;
     p.tcap = w.tcap;
     p.split_deg = split_degree(g, bt);
@@ -397,7 +416,7 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     const unsigned aux_grid = (unsigned)g->sm_count * 8 / conc + 1;
     CK(cudaEventRecord(w.ev[0], s), "event");
     init_run_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, g->n, source, p.ctl, p.bk, p.ring, w.cap, h0,
-                                                    p.expanded);
+                                                    p.expanded, p.filt);
     CK(cudaGetLastError(), "init kernel launch");
     CK(cudaEventRecord(w.ev[1], s), "event");
     void* args[] = {(void*)&p};
@@ -511,6 +530,11 @@ void accumulate(sssp_graph* g, Workspace& w, const Ctl& c, int bits) {
     st.reachable += c.reach_v;
     st.reach_edges += c.reach_e;
     st.max_dist = std::max<uint64_t>(st.max_dist, c.max_dist);
+    if (!g->f32 && c.max_dist) {  // resolution of the 16-bit filter for the next run on this graph
+        unsigned sh = 0;
+        while (sh < 48 && (c.max_dist >> sh) >= 60000ull) ++sh;
+        g->filt_shift_hint = sh + 1;  // stored +1 (0 = no run yet)
+    }
     st.init_delta_log2 = w.last_k0;
     st.final_delta_log2 = g->opts.algorithm == SSSP_ALGO_NEAR_FAR ? w.last_k0 : meta_k(c.head.meta);
     st.head_switches += c.head_switches;

@@ -114,6 +114,8 @@ PERTURB = [
     dict(split_degree=5, flags=sssp.SSSP_FLAG_NO_LOCAL), dict(split_degree=0xFFFFFFFF),
     # warp-local continuation off / with a 1-item CTA-level cap; 1024-thread CTAs
     dict(flags=sssp.SSSP_FLAG_NO_WARP_LOCAL), dict(flags=sssp.SSSP_FLAG_WARP_LOCAL, local_max=1, grid_ctas=2), dict(block_threads=1024),
+    # relaxation filter on the 16-bit upper-bound array instead of dist itself
+    dict(flags=sssp.SSSP_FLAG_FILTER16), dict(flags=sssp.SSSP_FLAG_FILTER16, dist_bits=64),
 ]
 
 
@@ -386,3 +388,21 @@ def test_hub_split_star():
     for opt in (dict(), dict(split_degree=1000), dict(split_degree=1000, grid_ctas=2), dict(split_degree=0xFFFFFFFF)):
         st = check(g, 0, **opt)
         assert st["edges_relaxed"] >= st["reach_edges"]
+
+
+def test_filter16_resolution_change_keeps_results():
+    """The 16-bit filter's resolution is refitted from each run's largest distance; runs on
+    graphs whose distances exceed 65534 * 2^s (no bound -> plain atomic) and sources with very
+    different ranges on one handle stay bit-exact (D11)."""
+    g = gg.make("road", scale_down=8)
+    G = sssp.Graph.from_csr(g, flags=sssp.SSSP_FLAG_FILTER16)
+    for s in list(gg.config_sources("road", g, 3)) + [0]:
+        d = sssp.to_u64(G.run(int(s)))
+        assert np.array_equal(d, oracle.dijkstra(g, int(s))[0])
+    # a chain whose distances run far beyond 65534 * 2^s for small weights
+    n = 70000
+    ch = gg.from_arcs(n, [(i, i + 1, 1 + (i % 3)) for i in range(n - 1)] + [(0, n - 1, 10**9)])
+    H = sssp.Graph.from_csr(ch, flags=sssp.SSSP_FLAG_FILTER16)
+    for _ in range(2):
+        d = sssp.to_u64(H.run(0))
+        assert np.array_equal(d, oracle.dijkstra(ch, 0)[0])
