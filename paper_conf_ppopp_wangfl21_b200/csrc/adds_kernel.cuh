@@ -763,6 +763,9 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         // Tiny batches (latency regime, road-like graphs) skip the L2 filter load.
         {
             const bool tiny = E <= (unsigned)BT;
+            // static slices (dynamic 32*EPT-arc chunks from a shared counter measured
+            // neutral on RMAT/ER, profiles/r01_sweeps.md §14)
+            constexpr unsigned kChunk = 32u * EPT;
             const unsigned per = (E + kWarps - 1) / kWarps;
             const unsigned slice = (per + 31) / 32 * 32;  // small batches spread over many warps
             const unsigned wb = warp * slice;
@@ -803,7 +806,6 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         if (want && pos < kWQ) {
                             s_wqv[wq0 + pos] = v;
                             s_wqd[wq0 + pos] = (DistT)ndv;
-                            if (!(p.exp & 1u)) prefetch_l1(p.off + v);  // the next hop reads this row from L1
                             kept = true;
                         }
                         const unsigned nn = wq_n + __popc(wm);
@@ -935,13 +937,13 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     emit(push[j] && !kept, a[j].x, nd[j], o);
                 }
             };
-            if (PIPE && we > wb + 32 * EPT) {
+            if (PIPE && we > wb + kChunk) {
                 // software pipeline: round r+1's owners and arc loads are issued before
                 // round r's gathers and atomics
                 unsigned own_n[EPT];
                 uint2 a_n[EPT];
-                fetch(wb, own_n, a_n);
-                for (unsigned base = wb; base < we; base += 32 * EPT) {
+                if (wb < we) fetch(wb, own_n, a_n);
+                for (unsigned base = wb; base < we;) {
                     unsigned own[EPT];
                     uint2 a[EPT];
 #pragma unroll
@@ -949,11 +951,13 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         own[j] = own_n[j];
                         a[j] = a_n[j];
                     }
-                    if (base + 32 * EPT < we) fetch(base + 32 * EPT, own_n, a_n);
+                    const unsigned nxt = base + kChunk;
+                    if (nxt < we) fetch(nxt, own_n, a_n);
                     body(base, own, a);
+                    base = nxt;
                 }
             } else {
-                for (unsigned base = wb; base < we; base += 32 * EPT) {
+                for (unsigned base = wb; base < we; base += kChunk) {
                     unsigned own[EPT];
                     uint2 a[EPT];
                     fetch(base, own, a);
@@ -983,21 +987,15 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
                 __syncwarp();
                 wq_n = st0;
-                // no stale re-check: the child was improved by this warp a hop ago (a
-                // superseded child only costs a redundant relaxation), so the hop waits on
-                // the L1-prefetched row alone
+                // stale re-check with the row loads (one round trip): skipping it expands
+                // superseded children and measured 1.7x -> 3.2x work on ROAD
                 unsigned long long b = 0, e = 0;
-                bool lv = has;
+                bool lv = false;
                 if (has) {
-                    if (p.exp & 1u) {  // A/B: previous hop shape (stale re-check, L2 row loads)
-                        const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
-                        b = ld_stream_u64(p.off + v, pol_stream);
-                        e = ld_stream_u64(p.off + v + 1, pol_stream);
-                        lv = cur >= dv;
-                    } else {
-                        b = ld_ca_u64(p.off + v);
-                        e = ld_ca_u64(p.off + v + 1);
-                    }
+                    const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
+                    b = ld_stream_u64(p.off + v, pol_stream);
+                    e = ld_stream_u64(p.off + v + 1, pol_stream);
+                    lv = cur >= dv;
                 }
                 const bool big = lv && (e - b) > kWDeg;
                 emit(big, v, dv, 0u);  // long rows: back to the head bucket through the ring

@@ -261,13 +261,6 @@ __device__ __forceinline__ void cp_async_8(unsigned sdst, const void* gsrc, unsi
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
-// non-blocking L1 prefetch of a read-only line (row offsets of a child kept for the next hop)
-__device__ __forceinline__ void prefetch_l1(const void* p) { asm volatile("prefetch.global.L1 [%0];" ::"l"(p)); }
-__device__ __forceinline__ unsigned long long ld_ca_u64(const unsigned long long* a) {
-    unsigned long long r;
-    asm volatile("ld.global.ca.u64 %0, [%1];" : "=l"(r) : "l"(a));
-    return r;
-}
 // non-blocking L2 prefetch (no register result, nothing waits on it)
 __device__ __forceinline__ void prefetch_l2(const void* p) {
     asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(p));
