@@ -85,6 +85,11 @@ typedef enum sssp_status {
                                      (tools/l2_residency_bench.cu) it shrinks the normal L2 and LOWERS
                                      random-gather throughput (213 vs 263 G/s next to a 4 GB stream) */
 
+/* Worker granularity (options.worker) */
+#define SSSP_WORKER_AUTO 0u
+#define SSSP_WORKER_CTA 1u
+#define SSSP_WORKER_WARP 2u
+
 /* Algorithms (options.algorithm) */
 #define SSSP_ALGO_ADDS 0u
 #define SSSP_ALGO_NEAR_FAR 1u
@@ -151,7 +156,12 @@ typedef struct sssp_options {
                                   chunks that idle CTAs claim before bucket items (charged to the
                                   vertex's bucket, so the head cannot pass it early); 0 = auto
                                   (8 x CTA size), UINT32_MAX = off */
-    uint32_t reserved2[2];
+    uint32_t worker;           /* unit of work of the ADDS persistent kernel: SSSP_WORKER_AUTO (0, = CTA),
+                                  SSSP_WORKER_CTA (a CTA claims up to a CTA-sized batch, expands it
+                                  cooperatively and keeps head-bucket children on chip) or
+                                  SSSP_WORKER_WARP (ablation: every warp is an independent worker with
+                                  up to 32 items and no CTA barrier; measured slower, D12) */
+    uint32_t reserved2[1];
 } sssp_options;
 
 typedef struct sssp_stats {
@@ -177,7 +187,7 @@ typedef struct sssp_stats {
     uint32_t status;             /* sssp_status of the last run (for SSSP_FLAG_ASYNC) */
     float batch_ms;              /* device time of the whole call on the caller's stream (CUDA events) */
     uint32_t concurrency;        /* sources that were in flight at once */
-    uint32_t reserved[1];
+    uint32_t worker;             /* SSSP_WORKER_CTA or SSSP_WORKER_WARP: the worker granularity that ran */
 } sssp_stats;
 
 /* One Delta-controller sample (written at each head-bucket switch and at each

@@ -37,6 +37,9 @@ SSSP_FLAG_ADAPT_ACTIVE = 0x40
 SSSP_FLAG_NO_WARP_LOCAL = 0x80
 SSSP_FLAG_WARP_LOCAL = 0x100
 SSSP_FLAG_FILTER16 = 0x200
+SSSP_WORKER_AUTO = 0
+SSSP_WORKER_CTA = 1
+SSSP_WORKER_WARP = 2
 PROFILE_FIELDS = ["cyc_claim", "cyc_idle", "cyc_pop", "cyc_scan", "cyc_rounds", "cyc_flush", "cyc_complete",
                   "cyc_total", "n_ring_batches", "n_local_batches", "n_idle", "n_flush", "n_rounds", "n_ctas",
                   "cyc_window", "n_windows"]
@@ -75,7 +78,7 @@ class sssp_options(ctypes.Structure):
         ("batch_min", ctypes.c_uint32), ("timeout_ms", ctypes.c_uint32), ("trace_capacity", ctypes.c_uint32),
         ("active_init", ctypes.c_uint32), ("local_max", ctypes.c_uint32), ("max_backoff_ns", ctypes.c_uint32),
         ("startup_permille", ctypes.c_uint32), ("concurrent_sources", ctypes.c_uint32),
-        ("algorithm", ctypes.c_uint32), ("split_degree", ctypes.c_uint32), ("reserved2", ctypes.c_uint32 * 2),
+        ("algorithm", ctypes.c_uint32), ("split_degree", ctypes.c_uint32), ("worker", ctypes.c_uint32), ("reserved2", ctypes.c_uint32 * 1),
     ]
 
 
@@ -88,7 +91,7 @@ class sssp_stats(ctypes.Structure):
         ("dist_bits", ctypes.c_uint32), ("grid_ctas", ctypes.c_uint32), ("block_threads", ctypes.c_uint32),
         ("runs", ctypes.c_uint32), ("trace_entries", ctypes.c_uint32), ("kernel_ms", ctypes.c_float),
         ("total_ms", ctypes.c_float), ("status", ctypes.c_uint32), ("batch_ms", ctypes.c_float),
-        ("concurrency", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 1),
+        ("concurrency", ctypes.c_uint32), ("worker", ctypes.c_uint32),
     ]
 
 

@@ -477,11 +477,11 @@ __device__ unsigned spawn_chunks(const Params<DistT>& p, unsigned v, unsigned lo
     for (unsigned c = 1; c <= extra; ++c) {
         const unsigned long long idx = t0 + c - 1;
         SplitTask* tp = p.tasks + (idx & (p.tcap - 1));
-        if (idx >= p.tcap) {  // the previous lap's occupant is claimed: wait for its reader to clear it
-            unsigned spins = 0;
-            while (ld_relaxed_u32(&tp->len) != 0)
-                if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) return S;
-        }
+        // take the slot (free -> busy); it is still occupied while the previous lap's
+        // chunk has not been read
+        unsigned spins = 0;
+        while (atomicCAS(&tp->len, 0u, kLenBusy) != 0u)
+            if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) return S;
         tp->beg = b + (unsigned long long)c * S;
         tp->d = d;
         tp->v = v;
@@ -494,6 +494,20 @@ __device__ unsigned spawn_chunks(const Params<DistT>& p, unsigned v, unsigned lo
     }
     atomicAdd(&p.bk[kSplitQ].avail.v, (unsigned long long)extra);
     return S;
+}
+
+// Take a published chunk (CAS len -> reading, acquire); returns its length, or 0
+// if the run was aborted while waiting.  The caller reads the payload and frees
+// the slot with a release store of 0 (common.cuh, kLenReading).
+template <typename DistT>
+__device__ __forceinline__ unsigned take_chunk(const Params<DistT>& p, SplitTask* tp) {
+    unsigned spins = 0;
+    for (;;) {
+        const unsigned len = ld_relaxed_u32(&tp->len);
+        if (len != 0u && len != kLenBusy && len != kLenReading && cas_acquire_u32(&tp->len, len, kLenReading) == len)
+            return len;
+        if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) return 0u;
+    }
 }
 
 // --------------------------------------------------------------- shared memory
@@ -656,15 +670,13 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             // a hub-split chunk: one vertex, len arcs, charged to the slot it carries
             if (tid == 0) {
                 SplitTask* tp = p.tasks + (s_idx & (p.tcap - 1));
-                unsigned len, spins = 0;
                 s_slot = 0;
-                while ((len = ld_acquire_u32(&tp->len)) == 0)
-                    if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;
+                const unsigned len = take_chunk(p, tp);
                 if (len) {
                     const unsigned long long b = __ldcg(&tp->beg), d = __ldcg(&tp->d);
                     const unsigned v = __ldcg(&tp->v);
                     s_slot = __ldcg(&tp->slot);
-                    st_relaxed_u32(&tp->len, 0u);  // clear behind the read
+                    st_release_u32(&tp->len, 0u);  // free the slot after the read
                     const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
                     if (cur >= d) {  // stale chunks (v improved since) are dropped
                         deg = len;
@@ -682,10 +694,9 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 const unsigned long long idx = (s_idx + tid) & (p.cap - 1);
                 char* sp = p.ring + ((size_t)slot * p.cap + idx) * IT::kBytes;
                 unsigned spins = 0;
-                while (!(loaded = IT::load(sp, v, d))) {  // reserved, store not landed yet
-                    if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;  // aborted run
+                while (!(loaded = IT::take(sp, v, d, spins++ == 0))) {  // reserved, put not landed yet
+                    if ((spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;  // aborted run
                 }
-                if (loaded) IT::clear(sp);
             } else {
                 v = s_lv[tid];
                 d = (unsigned long long)s_ld[tid];
@@ -875,17 +886,9 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         b0 = __shfl_sync(peers, b0, pl);
                         const unsigned long long idx = b0 + __popc(peers & lt_mask);
                         char* sp = p.ring + ((size_t)sl * p.cap + (idx & (p.cap - 1))) * IT::kBytes;
-                        bool ok = true;
-                        if (idx >= p.cap) {
-                            unsigned spins = 0;
-                            while (!IT::empty(sp)) {
-                                if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) {
-                                    ok = false;
-                                    break;
-                                }
-                            }
-                        }
-                        if (ok) IT::store(sp, IT::make(v, ndv));
+                        unsigned spins = 0;  // occupied while the previous lap's item is unread
+                        while (!IT::put(sp, IT::make(v, ndv)))
+                            if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) break;
                         __syncwarp(peers);
                         if (lane == pl) atomicAdd(&p.bk[sl].avail.v, (unsigned long long)__popc(peers));
                     }
@@ -1082,17 +1085,9 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     const unsigned sl = (hs + o) & nbm;
                     const unsigned long long idx = s_base[o] + s_rank[i];
                     char* sp = p.ring + ((size_t)sl * p.cap + (idx & (p.cap - 1))) * IT::kBytes;
-                    bool ok = true;
-                    if (idx >= p.cap) {  // wait for the previous lap's reader to clear it
-                        unsigned spins = 0;
-                        while (!IT::empty(sp)) {
-                            if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) {
-                                ok = false;
-                                break;
-                            }
-                        }
-                    }
-                    if (ok) IT::store(sp, s_items[i]);
+                    unsigned spins = 0;  // occupied while the previous lap's item is unread
+                    while (!IT::put(sp, s_items[i]))
+                        if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) break;
                 }
                 __syncthreads();
                 if (warp == 0 && lane < (int)p.nb) {

@@ -56,7 +56,15 @@ struct alignas(32) SplitTask {
     unsigned slot;
     unsigned pad_;
 };
-constexpr uint32_t kSplitQ = kMaxBuckets;  // index of the split queue's counters
+constexpr uint32_t kSplitQ = kMaxBuckets;
+// SplitTask.len states besides a real length: 0 = free, kLenBusy = a writer owns the
+// slot (payload being written), kLenReading = a reader owns it (payload being read).
+// Writers take a free slot by CAS 0 -> busy and publish with a release store of the
+// length; readers take a published slot by CAS len -> reading and free it with a
+// release store of 0 after reading, so no chunk is lost or taken twice even when
+// the queue laps with chunks claimed but not yet read.
+constexpr unsigned kLenBusy = 0xFFFFFFFFu;
+constexpr unsigned kLenReading = 0xFFFFFFFEu;  // index of the split queue's counters
 // In flight for bucket b = reserve + local - done.  The bucket is complete when
 // that is 0, and the run is finished when every bucket is complete
 // (exact quiescence, reading R11 of P:182): children are always counted (reserve
@@ -140,6 +148,14 @@ __device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
 }
 __device__ __forceinline__ void st_relaxed_u32(unsigned* p, unsigned v) {
     asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_u32(unsigned* p, unsigned v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned cas_acquire_u32(unsigned* p, unsigned cmp, unsigned val) {
+    unsigned r;
+    asm volatile("atom.acquire.gpu.global.cas.b32 %0, [%1], %2, %3;" : "=r"(r) : "l"(p), "r"(cmp), "r"(val) : "memory");
+    return r;
 }
 __device__ __forceinline__ unsigned ld_relaxed_u32(const unsigned* p) {
     unsigned v;
@@ -273,6 +289,14 @@ __device__ __forceinline__ unsigned lanemask_lt() {
 }
 
 // ------------------------------------------------------------ item formats
+// Ring slot protocol.  Claims hand out ring indices in order, but items are
+// published out of order (the avail gate counts items, not indices), so when a
+// bucket's circular array laps, a slot can be targeted by the writers -- and the
+// readers -- of two laps at once.  Plain stores/loads would then lose an item
+// (two writers both seeing the slot empty) or duplicate one (two readers both
+// seeing the same item).  Readers therefore take an item with one atomic
+// exchange (they own exactly what it returned) and writers fill a slot with one
+// CAS from empty (they wait while it is occupied).
 // 32-bit distances: one 64-bit word  (v | d << 32); empty = all ones (v = 2^32-1
 // is a reserved id).  A single 64-bit store is single-copy atomic, so writing
 // the item IS its publication: no write-completed counter and no fence per item
@@ -300,6 +324,22 @@ struct ItemT<uint32_t> {
     }
     __device__ __forceinline__ static void store(void* slot, Raw r) { st_relaxed_u64((unsigned long long*)slot, r); }
     __device__ __forceinline__ static void clear(void* slot) { st_relaxed_u64((unsigned long long*)slot, ~0ull); }
+    // Ownership-transferring ring ops (see "Ring slot protocol" above): take() empties
+    // the slot with one exchange and owns whatever it returned; put() fills an empty
+    // slot with one CAS.  Two writers of different laps, or two readers of different
+    // laps, can therefore never both succeed on one slot.
+    // (the claimer usually finds its item already there: exchange first, one round
+    // trip; an exchange of empty with empty is harmless; spin on plain loads after)
+    __device__ __forceinline__ static bool take(void* slot, uint32_t& v, unsigned long long& d, bool first) {
+        if (!first && ld_relaxed_u64((const unsigned long long*)slot) == ~0ull) return false;
+        const unsigned long long x = atomicExch((unsigned long long*)slot, ~0ull);
+        v = (uint32_t)x;
+        d = x >> 32;
+        return x != ~0ull;
+    }
+    __device__ __forceinline__ static bool put(void* slot, Raw r) {
+        return atomicCAS((unsigned long long*)slot, ~0ull, r) == ~0ull;
+    }
 };
 
 template <>
@@ -323,6 +363,37 @@ struct ItemT<unsigned long long> {
     }
     __device__ __forceinline__ static void store(void* slot, Raw r) { st_relaxed_v2u64(slot, r.v, r.d); }
     __device__ __forceinline__ static void clear(void* slot) { st_relaxed_v2u64(slot, ~0ull, ~0ull); }
+    __device__ __forceinline__ static bool take(void* slot, uint32_t& v, unsigned long long& d, bool first) {
+        unsigned long long a, b;
+        if (!first) {
+            ld_relaxed_v2u64(slot, a, b);
+            if (a == ~0ull && b == ~0ull) return false;  // empty (a put is one 128-bit CAS)
+        }
+        asm volatile(
+            "{\n\t.reg .b128 d, x;\n\t"
+            "mov.b128 x, {%2, %3};\n\t"
+            "atom.relaxed.gpu.global.exch.b128 d, [%4], x;\n\t"
+            "mov.b128 {%0, %1}, d;\n\t}"
+            : "=l"(a), "=l"(b)
+            : "l"(~0ull), "l"(~0ull), "l"(slot)
+            : "memory");
+        v = (uint32_t)a;
+        d = b;
+        return !(a == ~0ull && b == ~0ull);
+    }
+    __device__ __forceinline__ static bool put(void* slot, Raw r) {
+        unsigned long long o0, o1;
+        asm volatile(
+            "{\n\t.reg .b128 d, b, c;\n\t"
+            "mov.b128 b, {%2, %3};\n\t"
+            "mov.b128 c, {%4, %5};\n\t"
+            "atom.relaxed.gpu.global.cas.b128 d, [%6], b, c;\n\t"
+            "mov.b128 {%0, %1}, d;\n\t}"
+            : "=l"(o0), "=l"(o1)
+            : "l"(~0ull), "l"(~0ull), "l"(r.v), "l"(r.d), "l"(slot)
+            : "memory");
+        return o0 == ~0ull && o1 == ~0ull;
+    }
 };
 
 template <typename DistT>

@@ -13,6 +13,7 @@
 
 #include "../../include/sssp.h"
 #include "adds_kernel.cuh"
+#include "adds_warp_kernel.cuh"
 #include "aux_kernels.cuh"
 #include "nearfar_kernel.cuh"
 #include "bucket_map.h"
@@ -84,7 +85,7 @@ struct Workspace {
     DevBuf nf_piles, nf_cnt;            // Near-Far ablation: 4 pile buffers + counters
     unsigned long long nf_cap = 0;
     int nf_item_bytes = 0;
-    uint32_t last_grid = 0, last_block = 0, last_k0 = 0;
+    uint32_t last_grid = 0, last_block = 0, last_k0 = 0, last_worker = 0;
     void release() {
         dist.release();
         ring.release();
@@ -158,6 +159,7 @@ sssp_status check_options(const sssp_options& o) {
     if (o.waste_lo_permille > 1000 || o.waste_hi_permille > 1000) return fail(SSSP_ERR_INVALID_ARGUMENT, "waste permille");
     if (o.concurrent_sources > 64) return fail(SSSP_ERR_INVALID_ARGUMENT, "concurrent_sources > 64");
     if (o.algorithm > SSSP_ALGO_NEAR_FAR) return fail(SSSP_ERR_INVALID_ARGUMENT, "algorithm");
+    if (o.worker > SSSP_WORKER_WARP) return fail(SSSP_ERR_INVALID_ARGUMENT, "worker");
     return SSSP_OK;
 }
 
@@ -202,6 +204,28 @@ KVariant persistent_variant(int bits, int bt, bool f32) {
     return kvar<unsigned long long, 256>();
 }
 
+// Warp-granular worker (adds_warp_kernel.cuh): 512-thread CTAs, 2 per SM, EPT 4.
+template <typename DistT, bool kF = false>
+KVariant wvar() {
+    return KVariant{(void*)adds_warp_kernel<DistT, 512, 4, 2, kF>, (512 / 32) * sizeof(WarpSmem<DistT>)};
+}
+KVariant warp_variant(int bits, bool f32) {
+    if (f32) return wvar<uint32_t, true>();
+    return bits == 32 ? wvar<uint32_t>() : wvar<unsigned long long>();
+}
+// Which worker runs (D12).  The warp worker (no CTA barriers) was the
+// hypothesis for the throughput regime; measured on B200 it is slower on every
+// config (ER 16.3 vs 11.8 ms, RMAT 7.6 vs 6.7, ROAD 130 vs 44: 16x more claimers
+// on the same bucket counters, and per-warp batches of 32 items pay the claim
+// round trips 16x as often), so AUTO = CTA and the warp worker is an ablation.
+// SSSP_KVAR=8 / 9 force warp / CTA (A/B on one box).
+bool use_warp_worker(const sssp_graph* g) {
+    const char* e = std::getenv("SSSP_KVAR");
+    if (e && std::atoi(e) == 8) return true;
+    if (e && std::atoi(e) == 9) return false;
+    return g->opts.worker == SSSP_WORKER_WARP;
+}
+
 unsigned long long default_cap(const sssp_graph* g) {
     if (g->opts.ring_items) return next_pow2(std::max<unsigned long long>(g->opts.ring_items, 64ull));
     return next_pow2(std::max<unsigned long long>((unsigned long long)g->n, 1ull << 16));
@@ -221,7 +245,9 @@ sssp_status ensure_ring(sssp_graph* g, Workspace& w, int item_bytes, unsigned lo
 
 unsigned split_degree(const sssp_graph* g, unsigned bt) {
     if (g->opts.split_degree == 0xFFFFFFFFu) return 0u;
-    return g->opts.split_degree ? g->opts.split_degree : 8u * bt;
+    // (chunk lengths must stay below the queue's slot-state markers, common.cuh)
+    if (g->opts.split_degree) return std::min(g->opts.split_degree, 1u << 31);
+    return 8u * bt;  // warp worker: bt = 128 -> 1024 arcs
 }
 
 // Hub-split chunk queue: enough entries for every arc of the graph in chunks of
@@ -393,7 +419,9 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
                        unsigned k0, unsigned conc) {
     unsigned bt = g->opts.block_threads ? g->opts.block_threads : 512;
     if (kF && bt != 256) bt = 512;  // float variants are built for 256/512-thread CTAs
-    const KVariant kv = persistent_variant(bits, (int)bt, kF);
+    const bool warp_worker = use_warp_worker(g);
+    if (warp_worker) bt = 512;
+    const KVariant kv = warp_worker ? warp_variant(bits, kF) : persistent_variant(bits, (int)bt, kF);
     void* fn = kv.fn;
     CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kv.smem), "smem attribute");
     int occ = 0;
@@ -412,6 +440,14 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     const unsigned span = kF ? heuristic_k(g) : g->heur_k_span;
     Head h0{0ull, pack_meta(0, k, A0, std::min(k, span), 0)};
     Params<DistT> p = make_params<DistT>(g, w, grid, bt, k_max, conc);
+    if (warp_worker) {
+        // a warp claims up to 32 items; split hubs into 8 rounds of 32 x EPT arcs
+        unsigned sh = 0;
+        while ((1u << (sh + 1)) <= grid * (bt / 32)) ++sh;
+        p.share_shift = sh > 2 ? sh - 2 : 0;
+        p.split_deg = split_degree(g, 128);
+        p.prof = 0;
+    }
 
     const unsigned aux_grid = (unsigned)g->sm_count * 8 / conc + 1;
     CK(cudaEventRecord(w.ev[0], s), "event");
@@ -435,6 +471,7 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     CK(cudaMemcpyAsync(w.h_ctl, w.ctl.p, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "status copy");
     w.last_grid = grid;
     w.last_block = bt;
+    w.last_worker = warp_worker ? SSSP_WORKER_WARP : SSSP_WORKER_CTA;
     w.last_k0 = k;
     return SSSP_OK;
 }
@@ -492,6 +529,7 @@ sssp_status launch_nf(sssp_graph* g, Workspace& w, uint32_t source, void* out_de
     CK(cudaMemcpyAsync(w.h_ctl, w.ctl.p, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "status copy");
     w.last_grid = grid;
     w.last_block = 256;
+    w.last_worker = 0;
     w.last_k0 = std::min(k0, bits == 32 ? 31u : 62u);
     return SSSP_OK;
 }
@@ -542,6 +580,7 @@ void accumulate(sssp_graph* g, Workspace& w, const Ctl& c, int bits) {
     st.dist_bits = (uint32_t)bits;
     st.grid_ctas = w.last_grid;
     st.block_threads = w.last_block;
+    st.worker = w.last_worker;
     st.runs += 1;
     st.trace_entries = std::min<uint32_t>(c.trace_count, w.trace_alloc);
     float a = 0, b = 0;

@@ -53,6 +53,24 @@ def test_golden_fixtures_on_gpu(name):
     assert st["reachable"] == fx["V"] and st["reach_edges"] == fx["E"]
 
 
+@pytest.mark.parametrize("name", golden_names())
+def test_golden_fixtures_warp_worker(name):
+    fx = load_golden(name)
+    g = gg.from_arcs(fx["n"], fx["arcs"])
+    d, st = gpu_dist(g, fx["source"], worker=sssp.SSSP_WORKER_WARP)
+    assert [int(x) for x in d] == fx["dist"]
+    assert st["reachable"] == fx["V"] and st["reach_edges"] == fx["E"]
+    assert st["worker"] == sssp.SSSP_WORKER_WARP
+
+
+def test_worker_selection():
+    # AUTO = the CTA worker (measured faster everywhere, D12); WARP on request
+    rmat = gg.make("rmat", scale_down=10)
+    s = gg.config_sources("rmat", rmat, 1)[0]
+    assert check(rmat, s)["worker"] == sssp.SSSP_WORKER_CTA
+    assert check(rmat, s, worker=sssp.SSSP_WORKER_WARP)["worker"] == sssp.SSSP_WORKER_WARP
+
+
 def test_u32_overflow_reruns_in_64_bits():
     n = 10
     g = gg.from_arcs(n, [(i, i + 1, 0xFFFFFFFF) for i in range(n - 1)] + [(0, 5, 7)])
@@ -79,6 +97,7 @@ def test_random_small_graphs():
         arcs = list(zip(rng.integers(0, n, m), rng.integers(0, n, m), rng.integers(0, wmax, m, endpoint=True)))
         g = gg.from_arcs(n, arcs)
         check(g, int(rng.integers(0, n)))
+        check(g, int(rng.integers(0, n)), worker=sssp.SSSP_WORKER_WARP)
 
 
 def test_config_grid64():
@@ -116,6 +135,16 @@ PERTURB = [
     dict(flags=sssp.SSSP_FLAG_NO_WARP_LOCAL), dict(flags=sssp.SSSP_FLAG_WARP_LOCAL, local_max=1, grid_ctas=2), dict(block_threads=1024),
     # relaxation filter on the 16-bit upper-bound array instead of dist itself
     dict(flags=sssp.SSSP_FLAG_FILTER16), dict(flags=sssp.SSSP_FLAG_FILTER16, dist_bits=64),
+    # worker granularity (D12): each worker forced on every graph, and the warp
+    # worker under the schedule extremes (one CTA, 64-bit, tiny rings, 1-arc / no hub
+    # chunks, 2 buckets, Delta = 1, tracing, static huge Delta)
+    dict(worker=sssp.SSSP_WORKER_WARP), dict(worker=sssp.SSSP_WORKER_CTA),
+    dict(worker=sssp.SSSP_WORKER_WARP, grid_ctas=1), dict(worker=sssp.SSSP_WORKER_WARP, dist_bits=64),
+    dict(worker=sssp.SSSP_WORKER_WARP, ring_items=64), dict(worker=sssp.SSSP_WORKER_WARP, split_degree=1),
+    dict(worker=sssp.SSSP_WORKER_WARP, split_degree=0xFFFFFFFF), dict(worker=sssp.SSSP_WORKER_WARP, num_buckets=2),
+    dict(worker=sssp.SSSP_WORKER_WARP, delta_mode=1, delta_init=1),
+    dict(worker=sssp.SSSP_WORKER_WARP, delta_mode=1, delta_init=1 << 30),
+    dict(worker=sssp.SSSP_WORKER_WARP, flags=sssp.SSSP_FLAG_TRACE),
 ]
 
 
@@ -239,8 +268,14 @@ def test_repeat_runs_deterministic_and_reusable():
 def test_full_size_config(config):
     g = gg.make(config)
     s = int(gg.config_sources(config, g, 1)[0])
-    st = check(g, s)
-    assert st["dist_bits"] == 32
+    ref, V, E = oracle.dijkstra(g, s)
+    # the bench's launch configuration (auto worker) and each worker forced
+    for worker in (sssp.SSSP_WORKER_AUTO, sssp.SSSP_WORKER_CTA, sssp.SSSP_WORKER_WARP):
+        d, st = gpu_dist(g, s, worker=worker)
+        bad = np.flatnonzero(d != ref)
+        assert bad.size == 0, f"worker={worker}: {bad.size} mismatches, first v={bad[:5]}"
+        assert st["reachable"] == V and st["reach_edges"] == E
+        assert st["dist_bits"] == 32
 
 
 def test_run_batch_distributed_single_rank():
