@@ -529,11 +529,14 @@ struct Smem {
     static constexpr size_t o_scan = o_rank + align16((size_t)kStage * 2);    // u32[BT]
     static constexpr size_t o_lv = o_scan + align16((size_t)BT * 4);          // u32[BT] kept children
     static constexpr size_t o_soff = o_lv + align16((size_t)BT * 4);          // u8[kStage]
-    // warp-local continuation queues: kWQ {vertex, distance} per warp
-    static constexpr int kWQ = 128;
+    // warp-local continuation queues: kWQ {vertex, distance, row begin, degree} per warp
+    // (the row is fetched when the child is found, so a hop starts with its arc loads)
+    static constexpr int kWQ = 96;
     static constexpr size_t o_wqv = o_soff + align16((size_t)kStage);         // u32[BT/32 * kWQ]
     static constexpr size_t o_wqd = o_wqv + align16((size_t)(BT / 32) * kWQ * 4);  // DistT[BT/32 * kWQ]
-    static constexpr size_t bytes = o_wqd + align16((size_t)(BT / 32) * kWQ * sizeof(DistT));
+    static constexpr size_t o_wqb = o_wqd + align16((size_t)(BT / 32) * kWQ * sizeof(DistT));  // u64[]
+    static constexpr size_t o_wqn = o_wqb + (size_t)(BT / 32) * kWQ * 8;      // u32[]
+    static constexpr size_t bytes = o_wqn + align16((size_t)(BT / 32) * kWQ * 4);
 };
 
 // --------------------------------------------------------------- kernel
@@ -541,7 +544,9 @@ struct Smem {
 // budget 65536 / (MINB * BT)), PIPE: the arc loads of a warp's next round are
 // issued before the current round's gathers/atomics (software pipeline: one
 // fewer dependent L2/HBM trip per round), kF: float32 weights (NEXT-3).
-template <typename DistT, int BT, int EPT, int MINB, bool PIPE, bool kF>
+// WLC: the warp-local continuation loop is compiled in (latency-regime graphs); the
+// throughput build leaves it out so its register allocation is not shaped by it.
+template <typename DistT, int BT, int EPT, int MINB, bool PIPE, bool kF, bool WLC = true>
 __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<DistT> p) {
     using IT = ItemT<DistT>;
     using Raw = typename IT::Raw;
@@ -562,6 +567,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     constexpr unsigned kWQ = (unsigned)L::kWQ;
     unsigned* s_wqv = (unsigned*)(smem + L::o_wqv);
     DistT* s_wqd = (DistT*)(smem + L::o_wqd);
+    unsigned long long* s_wqb = (unsigned long long*)(smem + L::o_wqb);
+    unsigned* s_wqn = (unsigned*)(smem + L::o_wqn);
     __shared__ unsigned s_wst[5];  // warp-local continuation: expanded, first, edges, stale, kept
 
     __shared__ unsigned s_cnt[kMaxBuckets];
@@ -658,7 +665,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         const unsigned lcap = got * 2 <= (unsigned)BT ? local_max : 0u;
         // warp-local continuation (same regime): a warp runs its own head-bucket
         // children hop after hop with no CTA barrier (D9)
-        const bool wlc = lcap != 0 && p.warp_local != 0;
+        const bool wlc = WLC && lcap != 0 && p.warp_local != 0;
 
         // ------------------------------------------------------------ pop + stale check
         const Head hd = s_head;
@@ -694,9 +701,10 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 const unsigned long long idx = (s_idx + tid) & (p.cap - 1);
                 char* sp = p.ring + ((size_t)slot * p.cap + idx) * IT::kBytes;
                 unsigned spins = 0;
-                while (!(loaded = IT::take(sp, v, d, spins++ == 0))) {  // reserved, put not landed yet
-                    if ((spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;  // aborted run
+                while (!(loaded = IT::load(sp, v, d))) {  // reserved, store not landed yet
+                    if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;  // aborted run
                 }
+                if (loaded) IT::clear(sp);  // the slot's one reader this run (D13)
             } else {
                 v = s_lv[tid];
                 d = (unsigned long long)s_ld[tid];
@@ -808,15 +816,24 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             // continuation), then in the CTA's next batch (warp-aggregated slot grabs)
             unsigned wq_n = 0;  // warp-uniform fill of this warp's queue
             const unsigned wq0 = (unsigned)warp * kWQ;
-            auto keep = [&](const bool want, const unsigned v, const unsigned long long ndv) -> bool {
+            // rb/rn: the child's row (begin, degree) when already fetched (has_row), else it
+            // is loaded here
+            auto keep = [&](const bool want, const unsigned v, const unsigned long long ndv, const bool has_row,
+                            unsigned long long rb, unsigned rn) -> bool {
                 bool kept = false;
                 if (wlc) {
                     const unsigned wm = __ballot_sync(FULL, want);
                     if (wm) {
                         const unsigned pos = wq_n + __popc(wm & lt_mask);
                         if (want && pos < kWQ) {
+                            if (!has_row) {
+                                rb = ld_stream_u64(p.off + v, pol_stream);
+                                rn = (unsigned)(ld_stream_u64(p.off + v + 1, pol_stream) - rb);
+                            }
                             s_wqv[wq0 + pos] = v;
                             s_wqd[wq0 + pos] = (DistT)ndv;
+                            s_wqb[wq0 + pos] = rb;
+                            s_wqn[wq0 + pos] = rn;
                             kept = true;
                         }
                         const unsigned nn = wq_n + __popc(wm);
@@ -877,18 +894,13 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         if (lane == pl) {
                             const unsigned c = (unsigned)__popc(peers);
                             b0 = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
-                            if (b0 + c > p.cap) {
-                                const unsigned long long cl = ld_relaxed_u64(&p.bk[sl].claim.v);
-                                if (b0 + c - p.cap > cl) atomicOr(&p.ctl->status, kStRingOverflow);
-                            }
+                            if (b0 + c > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
                             atomicAdd(&s_direct, c);
                         }
                         b0 = __shfl_sync(peers, b0, pl);
                         const unsigned long long idx = b0 + __popc(peers & lt_mask);
-                        char* sp = p.ring + ((size_t)sl * p.cap + (idx & (p.cap - 1))) * IT::kBytes;
-                        unsigned spins = 0;  // occupied while the previous lap's item is unread
-                        while (!IT::put(sp, IT::make(v, ndv)))
-                            if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) break;
+                        // the slot's one writer this run (D13); beyond cap the run is aborted
+                        if (idx < p.cap) IT::store(p.ring + ((size_t)sl * p.cap + idx) * IT::kBytes, IT::make(v, ndv));
                         __syncwarp(peers);
                         if (lane == pl) atomicAdd(&p.bk[sl].avail.v, (unsigned long long)__popc(peers));
                     }
@@ -936,7 +948,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 for (int j = 0; j < EPT; ++j) {
                     if (!__any_sync(FULL, push[j])) continue;
                     const unsigned o = push[j] ? bucket_of<kF>(nd[j], k, hd.h, p.nb) : 0u;
-                    const bool kept = keep(push[j] && o == 0, a[j].x, nd[j]);
+                    const bool kept = keep(push[j] && o == 0, a[j].x, nd[j], false, 0ull, 0u);
                     emit(push[j] && !kept, a[j].x, nd[j], o);
                 }
             };
@@ -978,37 +990,40 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             // completes after its warps' queues drain), so no counter is touched.
             // Rows longer than kWDeg go back through the ring (head bucket).
             constexpr unsigned kWDeg = 8u * EPT;
-            while (wq_n > 0) {
+            if constexpr (WLC) while (wq_n > 0) {
                 const unsigned take = wq_n < 32u ? wq_n : 32u;
                 const unsigned st0 = wq_n - take;
                 const bool has = lane < (int)take;
-                unsigned v = 0;
-                unsigned long long dv = kInf;
+                unsigned v = 0, deg = 0;
+                unsigned long long dv = kInf, b = 0;
                 if (has) {
                     v = s_wqv[wq0 + st0 + lane];
                     dv = (unsigned long long)s_wqd[wq0 + st0 + lane];
+                    b = s_wqb[wq0 + st0 + lane];
+                    deg = s_wqn[wq0 + st0 + lane];
                 }
                 __syncwarp();
                 wq_n = st0;
-                // stale re-check with the row loads (one round trip): skipping it expands
-                // superseded children and measured 1.7x -> 3.2x work on ROAD
-                unsigned long long b = 0, e = 0;
-                bool lv = false;
-                if (has) {
-                    const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
-                    b = ld_stream_u64(p.off + v, pol_stream);
-                    e = ld_stream_u64(p.off + v + 1, pol_stream);
-                    lv = cur >= dv;
-                }
-                const bool big = lv && (e - b) > kWDeg;
-                emit(big, v, dv, 0u);  // long rows: back to the head bucket through the ring
-                lv = lv && !big;
+                // long rows go back to the head bucket through the ring (their popper
+                // re-checks staleness)
+                const bool big = has && deg > kWDeg;
+                emit(big, v, dv, 0u);
+                bool lv = has && !big;
+                // the stale re-check is in flight together with the first arc loads (one
+                // round trip); skipping it expands superseded children (measured 1.7x ->
+                // 3.2x work on ROAD)
+                const unsigned long long cur = lv ? (unsigned long long)ld_keep(p.dist + v, pol_keep) : 0ull;
+                uint2 a[EPT];
+#pragma unroll
+                for (int j = 0; j < EPT; ++j)
+                    a[j] = lv && (unsigned)j < deg ? ld_stream_u2(p.adj + b + j, pol_stream) : make_uint2(0u, 0u);
+                lv = lv && cur >= dv;
                 bool fst = false;
                 if (lv && p.dynamic) {
                     const unsigned bit = 1u << (v & 31);
                     fst = (atomicOr(p.expanded + (v >> 5), bit) & bit) == 0;
                 }
-                const unsigned deg = lv ? (unsigned)(e - b) : 0u;
+                if (!lv) deg = 0;
                 const unsigned nl = (unsigned)__popc(__ballot_sync(FULL, lv));
                 const unsigned nf = (unsigned)__popc(__ballot_sync(FULL, fst));
                 const unsigned ns = (unsigned)__popc(__ballot_sync(FULL, has && !lv && !big));
@@ -1021,23 +1036,29 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     if (ns) atomicAdd(&s_wst[3], ns);
                 }
                 for (unsigned kk = 0; kk < maxdeg; kk += EPT) {
-                    uint2 a[EPT];
-                    unsigned long long nd[EPT];
+                    if (kk > 0) {
+#pragma unroll
+                        for (int j = 0; j < EPT; ++j)
+                            a[j] = kk + j < deg ? ld_stream_u2(p.adj + b + kk + j, pol_stream) : make_uint2(0u, 0u);
+                    }
+                    unsigned long long nd[EPT], rb[EPT], re[EPT];
                     DistT old[EPT];
                     bool push[EPT];
-#pragma unroll
-                    for (int j = 0; j < EPT; ++j)
-                        a[j] = kk + j < deg ? ld_stream_u2(p.adj + b + kk + j, pol_stream) : make_uint2(0u, 0u);
 #pragma unroll
                     for (int j = 0; j < EPT; ++j) {
                         push[j] = false;
                         old[j] = (DistT)0;
+                        rb[j] = re[j] = 0;
                         nd[j] = kk + j < deg ? relax_sum<kF>(dv, a[j].y) : kInf;
                         if (kk + j < deg) {
                             if (sum_unusable<kF>(nd[j], kInf)) {
                                 if (!kF) atomicOr(&p.ctl->status, kStDistOverflow);
                             } else {
+                                // the target's row is fetched in the same round trip as the
+                                // atomicMin: a kept child starts its hop with its arc loads
                                 old[j] = atomic_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
+                                rb[j] = ld_stream_u64(p.off + a[j].x, pol_stream);
+                                re[j] = ld_stream_u64(p.off + a[j].x + 1, pol_stream);
                                 push[j] = true;
                             }
                         }
@@ -1048,7 +1069,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         if (push[j] && p.filt) st_filt(p.filt + a[j].x, filt_enc(nd[j], p.filt_shift));
                         if (!__any_sync(FULL, push[j])) continue;
                         const unsigned o = push[j] ? bucket_of<kF>(nd[j], k, hd.h, p.nb) : 0u;
-                        const bool kept = keep(push[j] && o == 0, a[j].x, nd[j]);
+                        const bool kept = keep(push[j] && o == 0, a[j].x, nd[j], true, rb[j], (unsigned)(re[j] - rb[j]));
                         emit(push[j] && !kept, a[j].x, nd[j], o);
                     }
                 }
@@ -1072,10 +1093,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         // termination) is performed before this CTA's completion atomic
                         const unsigned long long b = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
                         s_base[lane] = b;
-                        if (b + c > p.cap) {  // lapping: previous occupants must be claimed
-                            const unsigned long long cl = ld_relaxed_u64(&p.bk[sl].claim.v);
-                            if (b + c - p.cap > cl) atomicOr(&p.ctl->status, kStRingOverflow);
-                        }
+                        if (b + c > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
                     }
                 }
                 __syncthreads();
@@ -1084,10 +1102,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     if (o == 0xFF) continue;  // hole left by a direct publication
                     const unsigned sl = (hs + o) & nbm;
                     const unsigned long long idx = s_base[o] + s_rank[i];
-                    char* sp = p.ring + ((size_t)sl * p.cap + (idx & (p.cap - 1))) * IT::kBytes;
-                    unsigned spins = 0;  // occupied while the previous lap's item is unread
-                    while (!IT::put(sp, s_items[i]))
-                        if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) break;
+                    // the slot's one writer this run (D13); beyond cap the run is aborted
+                    if (idx < p.cap) IT::store(p.ring + ((size_t)sl * p.cap + idx) * IT::kBytes, s_items[i]);
                 }
                 __syncthreads();
                 if (warp == 0 && lane < (int)p.nb) {

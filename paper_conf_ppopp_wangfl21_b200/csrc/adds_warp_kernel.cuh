@@ -115,9 +115,10 @@ __global__ void __launch_bounds__(BT, MINB) adds_warp_kernel(const Params<DistT>
             char* sp = p.ring + ((size_t)slot * p.cap + ix) * IT::kBytes;
             unsigned spins = 0;
             bool loaded;
-            while (!(loaded = IT::take(sp, v, d, spins++ == 0)))
-                if ((spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;
+            while (!(loaded = IT::load(sp, v, d)))
+                if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;
             if (loaded) {
+                IT::clear(sp);  // the slot's one reader this run (D13)
                 const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
                 const unsigned long long b = ld_stream_u64(p.off + v, pol_stream);
                 const unsigned long long e = ld_stream_u64(p.off + v + 1, pol_stream);
@@ -164,10 +165,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_warp_kernel(const Params<DistT>
                 const unsigned sl = (hs + lane) & nbm;
                 const unsigned long long b = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
                 S.base[lane] = b;
-                if (b + c > p.cap) {  // lapping: previous occupants must be claimed
-                    const unsigned long long cl = ld_relaxed_u64(&p.bk[sl].claim.v);
-                    if (b + c - p.cap > cl) atomicOr(&p.ctl->status, kStRingOverflow);
-                }
+                if (b + c > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
                 if (p.dynamic && lane == (int)nbm) atomicAdd(&p.ctl->g_clip, (unsigned long long)c);
             }
             if (p.dynamic && lane == 0) atomicAdd(&p.ctl->g_push, (unsigned long long)s_n);
@@ -176,10 +174,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_warp_kernel(const Params<DistT>
                 const unsigned o = S.soff[i];
                 const unsigned sl = (hs + o) & nbm;
                 const unsigned long long ix = S.base[o] + S.rank[i];
-                char* sp = p.ring + ((size_t)sl * p.cap + (ix & (p.cap - 1))) * IT::kBytes;
-                unsigned spins = 0;  // occupied while the previous lap's item is unread
-                while (!IT::put(sp, S.items[i]))
-                    if ((++spins & 255) == 0 && ld_relaxed_u32(&p.ctl->status)) break;
+                if (ix < p.cap) IT::store(p.ring + ((size_t)sl * p.cap + ix) * IT::kBytes, S.items[i]);  // D13
             }
             __syncwarp();
             if (c) {

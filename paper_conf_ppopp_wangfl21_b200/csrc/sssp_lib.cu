@@ -171,9 +171,11 @@ struct KVariant {
     void* fn;
     size_t smem;
 };
-template <typename DistT, int BT, bool kF = false, int EPT = 4, int MINB = 1024 / BT, bool PIPE = false>
+template <typename DistT, int BT, bool kF = false, int EPT = 4, int MINB = 1024 / BT, bool PIPE = false, bool WLC = true>
 KVariant kvar() {
-    return KVariant{(void*)adds_persistent_kernel<DistT, BT, EPT, MINB, PIPE, kF>, Smem<DistT, BT, EPT>::bytes};
+    // (without the warp-local loop the per-warp continuation queues are not allocated)
+    return KVariant{(void*)adds_persistent_kernel<DistT, BT, EPT, MINB, PIPE, kF, WLC>,
+                    WLC ? Smem<DistT, BT, EPT>::bytes : Smem<DistT, BT, EPT>::o_wqv};
 }
 // SSSP_KVAR (experiments): 0 default (= 1 for 32-bit 512-thread CTAs); 1 pipelined 512x2/SM EPT 4; 2 pipelined 512x1/SM EPT 8;
 // 3 pipelined 1024x1/SM EPT 4; 4 pipelined 512x1/SM EPT 4; 5 plain 512x1/SM EPT 8;
@@ -182,7 +184,7 @@ static int kvar_env() {
     const char* e = std::getenv("SSSP_KVAR");
     return e ? std::atoi(e) : 0;
 }
-KVariant persistent_variant(int bits, int bt, bool f32) {
+KVariant persistent_variant(int bits, int bt, bool f32, bool wlc) {
     if (f32) return bt == 256 ? kvar<uint32_t, 256, true>() : kvar<uint32_t, 512, true>();
     const int kv = kvar_env();
     if (bits == 32) {
@@ -194,7 +196,8 @@ KVariant persistent_variant(int bits, int bt, bool f32) {
         if (kv == 6) return kvar<uint32_t, 256, false, 8, 2, true>();
         if (bt == 128) return kvar<uint32_t, 128>();
         if (kv == 7) return kvar<uint32_t, 512>();  // 512 x 2/SM without the software pipeline (A/B)
-        if (bt == 512) return kvar<uint32_t, 512, false, 4, 2, true>();  // default: pipelined
+        if (bt == 512)  // default: pipelined; the warp-local loop only where it can run
+            return wlc ? kvar<uint32_t, 512, false, 4, 2, true>() : kvar<uint32_t, 512, false, 4, 2, true, false>();
         if (bt == 1024) return kvar<uint32_t, 1024>();
         return kvar<uint32_t, 256>();
     }
@@ -224,6 +227,12 @@ bool use_warp_worker(const sssp_graph* g) {
     if (e && std::atoi(e) == 8) return true;
     if (e && std::atoi(e) == 9) return false;
     return g->opts.worker == SSSP_WORKER_WARP;
+}
+
+// warp-local continuation (D10): on for road-like graphs (average degree <= 8) unless disabled
+bool warp_local_on(const sssp_graph* g) {
+    if (g->opts.flags & (SSSP_FLAG_NO_LOCAL | SSSP_FLAG_NO_WARP_LOCAL)) return false;
+    return (g->opts.flags & SSSP_FLAG_WARP_LOCAL) || g->m <= 8ull * g->n;
 }
 
 unsigned long long default_cap(const sssp_graph* g) {
@@ -342,8 +351,7 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
     // warp-local continuation pays on low-degree graphs (road-like: each lane's row fits
     // one or two rounds of EPT arcs); on ER (degree 32) it serialised what the ring spreads
     // over CTAs (measured +13 %), so it is on by default only for average degree <= 8
-    p.warp_local = (g->opts.flags & (SSSP_FLAG_NO_LOCAL | SSSP_FLAG_NO_WARP_LOCAL)) ? 0u
-                   : (g->opts.flags & SSSP_FLAG_WARP_LOCAL) || g->m <= 8ull * g->n ? 1u : 0u;
+    p.warp_local = warp_local_on(g) ? 1u : 0u;
     p.max_backoff_ns = g->opts.max_backoff_ns ? g->opts.max_backoff_ns : 2048u;
     p.prof = (g->opts.flags & SSSP_FLAG_PROFILE) ? 1u : 0u;
     p.expanded = (unsigned*)w.expanded.p;
@@ -421,7 +429,7 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     if (kF && bt != 256) bt = 512;  // float variants are built for 256/512-thread CTAs
     const bool warp_worker = use_warp_worker(g);
     if (warp_worker) bt = 512;
-    const KVariant kv = warp_worker ? warp_variant(bits, kF) : persistent_variant(bits, (int)bt, kF);
+    const KVariant kv = warp_worker ? warp_variant(bits, kF) : persistent_variant(bits, (int)bt, kF, warp_local_on(g));
     void* fn = kv.fn;
     CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kv.smem), "smem attribute");
     int occ = 0;
