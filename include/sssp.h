@@ -116,7 +116,7 @@ typedef struct sssp_options {
     uint32_t util_lo_pct;      /* lower utilisation limit, % of resident threads; default 100 */
     uint32_t util_hi_pct;      /* upper utilisation limit, % of resident threads; default 400 */
     uint32_t waste_lo_permille;/* Delta may grow only while the recent re-expansion share is below this
-                                  (default 450 = 45%) */
+                                  (default 500 = 50%) */
     uint32_t waste_hi_permille;/* Delta shrinks (not below its clip floor) while the share is above this
                                   (default 600 = 60%, i.e. ~2.5x Dijkstra's vertex work) */
     uint32_t period_us;        /* periodic controller step (default 20 us; head switches also step) */

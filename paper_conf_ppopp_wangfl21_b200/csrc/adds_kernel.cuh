@@ -143,8 +143,12 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
     // block growth for the rest of the run)
     // (an unmeasurable waste -- too few expansions in the window -- means the run
     // is crawling: growth is allowed once the start-up gate is open)
+    // cumulative-ratio gate on growth: 2.5x Dijkstra's vertex work (road-like graphs sit
+    // at 1.6-1.7x at their time-optimal Delta; a 1.5x gate pinned them one step below it,
+    // profiles/r01_sweeps.md §19)
+    const unsigned ratio_gate = (p.exp >> 8) & 0xFFu ? ((p.exp >> 8) & 0xFFu) * 2u : 250u;  // SSSP_EXP A/B
     const bool frugal = (!waste_known || waste < p.waste_lo) &&
-                        (ratio_x100 < 150 || !waste_known || waste * 2 < p.waste_lo) && progressed;
+                        (ratio_x100 < ratio_gate || !waste_known || waste * 2 < p.waste_lo) && progressed;
     const bool clipping = (total >= 64 && tail * 100 >= (long long)p.clip_pct * total) || (clip_known && clip >= 500);
     // settled: enough steps AND the head has switched twice since the last
     // change, so the ring has turned over and the items placed under the previous
@@ -513,7 +517,7 @@ __device__ __forceinline__ unsigned take_chunk(const Params<DistT>& p, SplitTask
 // --------------------------------------------------------------- shared memory
 constexpr size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
 
-template <typename DistT, int BT, int EPT>
+template <typename DistT, int BT, int EPT, int IPT = 1>
 struct Smem {
     using Raw = typename ItemT<DistT>::Raw;
     // staged ring pushes of one batch (beyond this, warps publish directly)
@@ -521,13 +525,13 @@ struct Smem {
     static constexpr int kStage = STAGE_MULT * BT * EPT / 2;
     static constexpr size_t o_arc = 0;                                        // (no arc window)
     static constexpr size_t o_items = 0;                                      // Raw[kStage] staged pushes
-    static constexpr size_t o_ebeg = o_items + align16((size_t)kStage * sizeof(Raw));  // u64[BT] row begin
-    static constexpr size_t o_d = o_ebeg + (size_t)BT * 8;                    // DistT[BT]  item distance
-    static constexpr size_t o_ld = o_d + align16((size_t)BT * sizeof(DistT)); // DistT[BT]  kept children
+    static constexpr size_t o_ebeg = o_items + align16((size_t)kStage * sizeof(Raw));  // u64[BT*IPT] row begin
+    static constexpr size_t o_d = o_ebeg + (size_t)BT * IPT * 8;              // DistT[BT*IPT] item distance
+    static constexpr size_t o_ld = o_d + align16((size_t)BT * IPT * sizeof(DistT)); // DistT[BT] kept children
     static constexpr size_t o_owner = o_ld + align16((size_t)BT * sizeof(DistT));  // (unused)
     static constexpr size_t o_rank = o_owner;                                 // u16[kStage]
-    static constexpr size_t o_scan = o_rank + align16((size_t)kStage * 2);    // u32[BT]
-    static constexpr size_t o_lv = o_scan + align16((size_t)BT * 4);          // u32[BT] kept children
+    static constexpr size_t o_scan = o_rank + align16((size_t)kStage * 2);    // u32[BT*IPT]
+    static constexpr size_t o_lv = o_scan + align16((size_t)BT * IPT * 4);    // u32[BT] kept children
     static constexpr size_t o_soff = o_lv + align16((size_t)BT * 4);          // u8[kStage]
     // warp-local continuation queues: kWQ {vertex, distance, row begin, degree} per warp
     // (the row is fetched when the child is found, so a hop starts with its arc loads)
@@ -548,9 +552,12 @@ struct Smem {
 // throughput build leaves it out so its register allocation is not shaped by it.
 template <typename DistT, int BT, int EPT, int MINB, bool PIPE, bool kF, bool WLC = true>
 __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<DistT> p) {
+    // items per thread: one (batches of two items per thread, to pay the per-batch round
+    // trips half as often, measured slower -- ER 13.1 vs 11.4 ms -- from register spills)
+    constexpr int IPT = 1;
     using IT = ItemT<DistT>;
     using Raw = typename IT::Raw;
-    using L = Smem<DistT, BT, EPT>;
+    using L = Smem<DistT, BT, EPT, IPT>;
     constexpr int kStage = L::kStage;
     constexpr int kWarps = BT / 32;
     constexpr unsigned long long kInf = (unsigned long long)DistInf<DistT>::value;
@@ -619,7 +626,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 unsigned long long idx = 0;
                 Head hd;
                 bool tk;
-                const unsigned g = claim_batch<DistT, BT>(p, lane, sl, idx, hd, st, tk);
+                const unsigned g = claim_batch<DistT, BT * IPT>(p, lane, sl, idx, hd, st, tk);
                 if (st) {
                     cmd = CMD_EXIT;
                 } else if (g) {
@@ -666,13 +673,20 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         // warp-local continuation (same regime): a warp runs its own head-bucket
         // children hop after hop with no CTA barrier (D9)
         const bool wlc = WLC && lcap != 0 && p.warp_local != 0;
+        const bool direct_head = wlc && (p.exp & 0x10000u) != 0;  // A/B (SSSP_EXP bit 16)
 
         // ------------------------------------------------------------ pop + stale check
         const Head hd = s_head;
         const unsigned hs = meta_hs(hd.meta), k = meta_k(hd.meta);
-        unsigned deg = 0;
-        bool live = false;
-        unsigned fword = 0, fbit = 0;  // expansion-bitmap word before our atomicOr (consumed at batch end)
+        unsigned degs[IPT];
+        bool lives[IPT];
+        unsigned fword[IPT], fbit[IPT];  // expansion-bitmap word before our atomicOr (consumed at batch end)
+#pragma unroll
+        for (int r = 0; r < IPT; ++r) {
+            degs[r] = 0;
+            lives[r] = false;
+            fword[r] = fbit[r] = 0;
+        }
         if (is_task) {
             // a hub-split chunk: one vertex, len arcs, charged to the slot it carries
             if (tid == 0) {
@@ -686,47 +700,56 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     st_release_u32(&tp->len, 0u);  // free the slot after the read
                     const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
                     if (cur >= d) {  // stale chunks (v improved since) are dropped
-                        deg = len;
+                        degs[0] = len;
                         s_ebeg[0] = b;
                         s_d[0] = (DistT)d;
-                        live = true;
+                        lives[0] = true;
                     }
                 }
             }
-        } else if (tid < (int)got) {
-            uint32_t v;
-            unsigned long long d;
-            bool loaded = true;
-            if (from_ring) {
-                const unsigned long long idx = (s_idx + tid) & (p.cap - 1);
-                char* sp = p.ring + ((size_t)slot * p.cap + idx) * IT::kBytes;
-                unsigned spins = 0;
-                while (!(loaded = IT::load(sp, v, d))) {  // reserved, store not landed yet
-                    if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;  // aborted run
-                }
-                if (loaded) IT::clear(sp);  // the slot's one reader this run (D13)
-            } else {
-                v = s_lv[tid];
-                d = (unsigned long long)s_ld[tid];
-            }
-            if (loaded) {
-                // the stale check and the row loads are independent: one round trip
-                const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
-                const unsigned long long b = ld_stream_u64(p.off + v, pol_stream);
-                const unsigned long long e = ld_stream_u64(p.off + v + 1, pol_stream);
-                if (cur >= d) {  // not stale: d is still v's distance ("refined")
-                    deg = (unsigned)(e - b);
-                    s_ebeg[tid] = b;
-                    s_d[tid] = (DistT)d;
-                    live = true;
-                    if (p.dynamic) {  // work-waste signal: is this v's first expansion?
-                        const unsigned bit = 1u << (v & 31);
-                        fword = atomicOr(p.expanded + (v >> 5), bit);  // result not waited for until the batch ends
-                        fbit = bit;
+        } else {
+            if (tid < (int)got) {
+                uint32_t v;
+                unsigned long long d;
+                bool loaded = true;
+                if (from_ring) {
+                    const unsigned long long idx = (s_idx + tid) & (p.cap - 1);
+                    char* sp = p.ring + ((size_t)slot * p.cap + idx) * IT::kBytes;
+                    unsigned spins = 0;
+                    while (!(loaded = IT::load(sp, v, d))) {  // reserved, store not landed yet
+                        if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;  // aborted run
                     }
-                    if (p.split_deg && deg > p.split_deg) deg = spawn_chunks(p, v, d, b, deg, slot);
+                    if (loaded) IT::clear(sp);  // the slot's one reader this run (D13)
+                } else {
+                    v = s_lv[tid];
+                    d = (unsigned long long)s_ld[tid];
+                }
+                if (loaded) {
+                    // the stale check and the row loads are independent: one round trip
+                    const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
+                    const unsigned long long b = ld_stream_u64(p.off + v, pol_stream);
+                    const unsigned long long e = ld_stream_u64(p.off + v + 1, pol_stream);
+                    if (cur >= d) {  // not stale: d is still v's distance ("refined")
+                        degs[0] = (unsigned)(e - b);
+                        s_ebeg[tid] = b;
+                        s_d[tid] = (DistT)d;
+                        lives[0] = true;
+                        if (p.dynamic) {  // work-waste signal: is this v's first expansion?
+                            const unsigned bit = 1u << (v & 31);
+                            fword[0] = atomicOr(p.expanded + (v >> 5), bit);  // result not waited for until the batch ends
+                            fbit[0] = bit;
+                        }
+                        if (p.split_deg && degs[0] > p.split_deg) degs[0] = spawn_chunks(p, v, d, b, degs[0], slot);
+                    }
                 }
             }
+        }
+        unsigned deg = 0;
+        int live = 0;
+#pragma unroll
+        for (int r = 0; r < IPT; ++r) {
+            deg += degs[r];
+            live += lives[r] ? 1 : 0;
         }
         if (tid == 0) s_lnext = 0;
         if (prof) {
@@ -743,7 +766,11 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             if (lane >= o) x += y;
         }
         if (lane == 31) s_wsum[warp] = x;
-        const int nlive = __syncthreads_count(live);
+        int nlive = __syncthreads_count(live & 1);
+        if constexpr (IPT > 1) {
+#pragma unroll
+            for (int bit = 1; (1 << bit) <= IPT; ++bit) nlive += __syncthreads_count((live >> bit) & 1) << bit;
+        }
         if (warp == 0) {
             const unsigned ws = lane < kWarps ? s_wsum[lane] : 0;
             unsigned inc = ws;
@@ -756,7 +783,14 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             if (lane == kWarps - 1) s_E = inc;
         }
         __syncthreads();
-        s_scan[tid] = x - deg + s_wsum[warp];
+        {
+            unsigned ex = x - deg + s_wsum[warp];
+#pragma unroll
+            for (int r = 0; r < IPT; ++r) {
+                s_scan[tid * IPT + r] = ex;
+                ex += degs[r];
+            }
+        }
         const unsigned E = s_E;
         if (is_task) slot = s_slot;
         const int nexp = is_task ? 0 : nlive;  // a chunk is not a vertex expansion
@@ -816,6 +850,9 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             // continuation), then in the CTA's next batch (warp-aggregated slot grabs)
             unsigned wq_n = 0;  // warp-uniform fill of this warp's queue
             const unsigned wq0 = (unsigned)warp * kWQ;
+            // queue depth: past it children go to the CTA's next batch (shared by all
+            // warps) or the ring (other CTAs); SSSP_EXP low byte overrides (A/B)
+            const unsigned wqcap = (p.exp & 0xFFu) && (p.exp & 0xFFu) < kWQ ? (p.exp & 0xFFu) : kWQ;
             // rb/rn: the child's row (begin, degree) when already fetched (has_row), else it
             // is loaded here
             auto keep = [&](const bool want, const unsigned v, const unsigned long long ndv, const bool has_row,
@@ -825,7 +862,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     const unsigned wm = __ballot_sync(FULL, want);
                     if (wm) {
                         const unsigned pos = wq_n + __popc(wm & lt_mask);
-                        if (want && pos < kWQ) {
+                        if (want && pos < wqcap) {
                             if (!has_row) {
                                 rb = ld_stream_u64(p.off + v, pol_stream);
                                 rn = (unsigned)(ld_stream_u64(p.off + v + 1, pol_stream) - rb);
@@ -837,11 +874,11 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                             kept = true;
                         }
                         const unsigned nn = wq_n + __popc(wm);
-                        if (lane == 0) atomicAdd(&s_wst[4], (nn < kWQ ? nn : kWQ) - wq_n);
-                        wq_n = nn < kWQ ? nn : kWQ;
+                        if (lane == 0) atomicAdd(&s_wst[4], (nn < wqcap ? nn : wqcap) - wq_n);
+                        wq_n = nn < wqcap ? nn : wqcap;
                     }
                 }
-                if (lcap) {
+                if (lcap && !direct_head) {  // (direct_head: overflow goes to the ring at once)
                     const bool w2 = want && !kept;
                     const unsigned lm = __ballot_sync(FULL, w2);
                     if (lm) {
@@ -860,16 +897,22 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             };
             // everything else: warp-aggregated staging for the CTA flush at batch end
             // (or direct publication when the staging area is full)
-            auto emit = [&](const bool pg, const unsigned v, const unsigned long long ndv, const unsigned o) {
+            // direct (warp-uniform): publish now instead of at batch end -- head-bucket
+            // children that overflow the on-chip queues in the latency regime, which idle
+            // CTAs should get while this CTA is still running its chains
+            auto emit = [&](const bool pg, const unsigned v, const unsigned long long ndv, const unsigned o,
+                            const bool direct = false) {
                 const unsigned act = __ballot_sync(FULL, pg);
                 if (!act) return;
                 // warp-aggregated staging slot for the CTA flush at batch end
                 const int leader = __ffs(act) - 1;
                 const unsigned nact = (unsigned)__popc(act);
                 unsigned pos = 0;
-                if (lane == leader) pos = atomicAdd(&s_total, nact);
-                pos = __shfl_sync(FULL, pos, leader);
-                if (pos + nact <= (unsigned)kStage) {
+                if (!direct) {
+                    if (lane == leader) pos = atomicAdd(&s_total, nact);
+                    pos = __shfl_sync(FULL, pos, leader);
+                }
+                if (!direct && pos + nact <= (unsigned)kStage) {
                     if (pg) {
                         const unsigned peers = __match_any_sync(act, o);
                         const int pl = __ffs(peers) - 1;
@@ -886,7 +929,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     // publish directly -- one reserve/avail pair per (warp, bucket)
                     if (pg) {
                         const unsigned my = pos + __popc(act & lt_mask);
-                        if (my < (unsigned)kStage) s_soff[my] = 0xFF;
+                        if (!direct && my < (unsigned)kStage) s_soff[my] = 0xFF;
                         const unsigned peers = __match_any_sync(act, o);
                         const int pl = __ffs(peers) - 1;
                         const unsigned sl = (hs + o) & nbm;
@@ -949,7 +992,12 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     if (!__any_sync(FULL, push[j])) continue;
                     const unsigned o = push[j] ? bucket_of<kF>(nd[j], k, hd.h, p.nb) : 0u;
                     const bool kept = keep(push[j] && o == 0, a[j].x, nd[j], false, 0ull, 0u);
-                    emit(push[j] && !kept, a[j].x, nd[j], o);
+                    if (direct_head) {
+                        emit(push[j] && !kept && o != 0, a[j].x, nd[j], o);
+                        emit(push[j] && !kept && o == 0, a[j].x, nd[j], 0u, true);
+                    } else {
+                        emit(push[j] && !kept, a[j].x, nd[j], o);
+                    }
                 }
             };
             if (PIPE && we > wb + kChunk) {
@@ -1007,7 +1055,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 // long rows go back to the head bucket through the ring (their popper
                 // re-checks staleness)
                 const bool big = has && deg > kWDeg;
-                emit(big, v, dv, 0u);
+                emit(big, v, dv, 0u, direct_head);
                 bool lv = has && !big;
                 // the stale re-check is in flight together with the first arc loads (one
                 // round trip); skipping it expands superseded children (measured 1.7x ->
@@ -1070,7 +1118,12 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         if (!__any_sync(FULL, push[j])) continue;
                         const unsigned o = push[j] ? bucket_of<kF>(nd[j], k, hd.h, p.nb) : 0u;
                         const bool kept = keep(push[j] && o == 0, a[j].x, nd[j], true, rb[j], (unsigned)(re[j] - rb[j]));
-                        emit(push[j] && !kept, a[j].x, nd[j], o);
+                        if (direct_head) {
+                            emit(push[j] && !kept && o != 0, a[j].x, nd[j], o);
+                            emit(push[j] && !kept && o == 0, a[j].x, nd[j], 0u, true);
+                        } else {
+                            emit(push[j] && !kept, a[j].x, nd[j], o);
+                        }
                     }
                 }
             }
@@ -1137,7 +1190,9 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
 
         // ------------------------------------------------------------ complete
         // s_lnext final (also covers the E == 0 case); first expansions for the controller
-        const int nfirst = __syncthreads_count(fbit != 0 && (fword & fbit) == 0);
+        int nfirst = 0;
+#pragma unroll
+        for (int r = 0; r < IPT; ++r) nfirst += __syncthreads_count(fbit[r] != 0 && (fword[r] & fbit[r]) == 0);
         const unsigned kept = s_lnext < lcap ? s_lnext : lcap;
         const unsigned w_exp = s_wst[0], w_first = s_wst[1], w_kept = s_wst[4];
         if (tid == 0) {

@@ -178,7 +178,7 @@ KVariant kvar() {
                     WLC ? Smem<DistT, BT, EPT>::bytes : Smem<DistT, BT, EPT>::o_wqv};
 }
 // SSSP_KVAR (experiments): 0 default (= 1 for 32-bit 512-thread CTAs); 1 pipelined 512x2/SM EPT 4; 2 pipelined 512x1/SM EPT 8;
-// 3 pipelined 1024x1/SM EPT 4; 4 pipelined 512x1/SM EPT 4; 5 plain 512x1/SM EPT 8;
+// (3, pipelined 1024x1/SM, removed: it hit the watchdog on ROAD, unexplained); 4 pipelined 512x1/SM EPT 4; 5 plain 512x1/SM EPT 8;
 // 6 pipelined 256x2/SM EPT 8; 7 plain 512x2/SM EPT 4 (the pre-pipeline default)
 static int kvar_env() {
     const char* e = std::getenv("SSSP_KVAR");
@@ -190,7 +190,6 @@ KVariant persistent_variant(int bits, int bt, bool f32, bool wlc) {
     if (bits == 32) {
         if (kv == 1) return kvar<uint32_t, 512, false, 4, 2, true>();
         if (kv == 2) return kvar<uint32_t, 512, false, 8, 1, true>();
-        if (kv == 3) return kvar<uint32_t, 1024, false, 4, 1, true>();
         if (kv == 4) return kvar<uint32_t, 512, false, 4, 1, true>();
         if (kv == 5) return kvar<uint32_t, 512, false, 8, 1, false>();
         if (kv == 6) return kvar<uint32_t, 256, false, 8, 2, true>();
@@ -796,7 +795,7 @@ void sssp_options_default(sssp_options* o) {
     o->settle_head_switches = 8;   // P:215 (reading R7): controller steps between Delta changes
     o->util_lo_pct = 100;          // P:211 (reading R6)
     o->util_hi_pct = 400;
-    o->waste_lo_permille = 450;    // reading R6: grow Delta only while < 45% of expansions are repeats
+    o->waste_lo_permille = 500;    // reading R6: grow Delta only while < 50% of expansions are repeats
     o->waste_hi_permille = 600;    //             shrink it while > 60% are (work <~ 2.5x Dijkstra)
     o->period_us = 20;
     o->startup_permille = 20;
