@@ -77,6 +77,10 @@ typedef enum sssp_status {
 #define SSSP_FLAG_FILTER16 0x200u     /* experiment (off by default, measured slower): filter relaxations
                                          with a 16-bit upper-bound array of dist (half its L2 footprint)
                                          instead of a load of dist itself; D11 */
+#define SSSP_FLAG_RELABEL 0x400u      /* force the locality relabeling of the graph at create time (vertices
+                                         renumbered by descending in-degree inside the library; inputs and
+                                         outputs stay in the caller's numbering; D15) */
+#define SSSP_FLAG_NO_RELABEL 0x800u   /* never relabel (default: relabel when max in-degree > 64 x average) */
 #define SSSP_FLAG_ADAPT_ACTIVE 0x40u  /* let the controller vary the number of active buckets;
                                         off by default: on our workloads it raised re-expansions */
 #define SSSP_FLAG_L2_PERSIST 0x20u /* reserve the L2 persisting set-aside for dist (raises the device-wide
@@ -292,6 +296,12 @@ sssp_status sssp_get_profile(sssp_graph *g, uint64_t *out, uint32_t cap, uint32_
  * D = m/n. */
 sssp_status sssp_graph_info(const sssp_graph *g, uint32_t *n, uint64_t *m, uint64_t *sum_w,
                             uint32_t *max_w, uint32_t *heuristic_delta_log2);
+
+/* Internal layout of the graph: *relabeled = 1 when the vertices were renumbered by
+ * descending in-degree at create time (D15: locality of the gathered /
+ * atomically updated distance array; sources and outputs always use the caller's
+ * numbering), *max_indeg = the largest in-degree.  Either pointer may be NULL. */
+sssp_status sssp_graph_layout(const sssp_graph *g, uint32_t *relabeled, uint32_t *max_indeg);
 
 /* The bucket ring's priority mapping (§5.4-5.5), exposed for unit
  * tests: the ring offset (0 = head ... B-1 = tail) that an item of distance d

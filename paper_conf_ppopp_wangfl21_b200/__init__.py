@@ -37,6 +37,8 @@ SSSP_FLAG_ADAPT_ACTIVE = 0x40
 SSSP_FLAG_NO_WARP_LOCAL = 0x80
 SSSP_FLAG_WARP_LOCAL = 0x100
 SSSP_FLAG_FILTER16 = 0x200
+SSSP_FLAG_RELABEL = 0x400
+SSSP_FLAG_NO_RELABEL = 0x800
 SSSP_WORKER_AUTO = 0
 SSSP_WORKER_CTA = 1
 SSSP_WORKER_WARP = 2
@@ -121,6 +123,7 @@ SIGNATURES = [
     ("sssp_get_trace", ctypes.c_int, [_P, _P, ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint32)]),
     ("sssp_get_profile", ctypes.c_int, [_P, _P, ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint32)]),
     ("sssp_graph_info", ctypes.c_int, [_P, _P, _P, _P, _P, _P]),
+    ("sssp_graph_layout", ctypes.c_int, [_P, _P, _P]),
     ("sssp_bucket_offset", ctypes.c_uint32, [ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_uint32]),
     ("sssp_status_string", ctypes.c_char_p, [ctypes.c_int]),
     ("sssp_last_error", ctypes.c_char_p, []),
@@ -301,7 +304,10 @@ class Graph:
         n, m, sw, mw, hk = ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_uint32(), ctypes.c_uint32()
         _check(lib().sssp_graph_info(self._h, ctypes.byref(n), ctypes.byref(m), ctypes.byref(sw), ctypes.byref(mw),
                                      ctypes.byref(hk)))
-        return {"n": n.value, "m": m.value, "sum_w": sw.value, "max_w": mw.value, "heuristic_delta_log2": hk.value}
+        rl, mi = ctypes.c_uint32(), ctypes.c_uint32()
+        _check(lib().sssp_graph_layout(self._h, ctypes.byref(rl), ctypes.byref(mi)))
+        return {"n": n.value, "m": m.value, "sum_w": sw.value, "max_w": mw.value, "heuristic_delta_log2": hk.value,
+                "relabeled": rl.value, "max_indeg": mi.value}
 
 
 def to_u64(t) -> np.ndarray:

@@ -550,7 +550,11 @@ struct Smem {
 // fewer dependent L2/HBM trip per round), kF: float32 weights (NEXT-3).
 // WLC: the warp-local continuation loop is compiled in (latency-regime graphs); the
 // throughput build leaves it out so its register allocation is not shaped by it.
-template <typename DistT, int BT, int EPT, int MINB, bool PIPE, bool kF, bool WLC = true>
+// CA: claim-ahead in the throughput regime -- warp 0 claims the next batch as soon as it
+// has streamed its own slice of the current one, so the claim round trips overlap the
+// other warps' streaming, the flush and the completion (held for the tail of one batch
+// only; claiming at the start of a batch held the claim too long, sweeps §7).
+template <typename DistT, int BT, int EPT, int MINB, bool PIPE, bool kF, bool WLC = true, bool CA = false>
 __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<DistT> p) {
     // items per thread: one (batches of two items per thread, to pay the per-batch round
     // trips half as often, measured slower -- ER 13.1 vs 11.4 ms -- from register spills)
@@ -581,7 +585,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     __shared__ unsigned s_cnt[kMaxBuckets];
     __shared__ unsigned long long s_base[kMaxBuckets];
     __shared__ unsigned s_wsum[kWarps];
-    __shared__ unsigned s_total, s_E, s_got, s_slot, s_lnext, s_direct, s_task;
+    __shared__ unsigned s_total, s_E, s_got, s_slot, s_lnext, s_direct, s_task, s_ahead;
     __shared__ int s_cmd;
     __shared__ unsigned long long s_idx;
     __shared__ Head s_head;
@@ -602,6 +606,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         s_total = 0;
         s_lnext = 0;
         s_direct = 0;
+        s_ahead = 0;
     }
     const bool prof = p.prof != 0 && tid == 0;
     const unsigned long long pol_stream = policy_evict_first();  // arcs, row offsets
@@ -618,6 +623,11 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             got = have_local;
             slot = s_slot;
             from_ring = false;
+        } else if (CA && s_ahead) {  // claimed ahead by warp 0 during the previous batch
+            got = s_got;
+            slot = s_slot;
+            from_ring = true;
+            is_task = s_task != 0;
         } else {
             // -------------------------------------------------------- claim
             if (warp == 0) {
@@ -808,6 +818,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         }
 
         __syncthreads();  // publishes s_scan / s_d / s_ebeg
+        if (CA && tid == 0) s_ahead = 0;  // every thread has read it (loop top)
         // ---------------------------------------------------- stream the batch's arcs
         // Warp w owns a contiguous slice of the batch's arc space and streams through
         // it with no CTA barrier (warps drift and keep the L1TEX queue busy); lanes
@@ -1125,6 +1136,26 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                             emit(push[j] && !kept, a[j].x, nd[j], o);
                         }
                     }
+                }
+            }
+        }
+        if constexpr (CA) {
+            // the batch's claim state (s_got/s_slot/s_idx/s_head/s_task) was consumed before
+            // the streaming barrier; kept children (which also use s_slot) need lcap != 0
+            if (warp == 0 && lcap == 0) {
+                unsigned sl = 0, st = 0;
+                unsigned long long idx = 0;
+                Head hd2;
+                bool tk;
+                const unsigned g = claim_batch<DistT, BT * IPT>(p, lane, sl, idx, hd2, st, tk);
+                if (lane == 0 && g) {
+                    s_got = g;
+                    s_slot = sl;
+                    s_idx = idx;
+                    s_head = hd2;
+                    s_task = tk ? 1u : 0u;
+                    s_ahead = 1;
+                    backoff = 0;
                 }
             }
         }

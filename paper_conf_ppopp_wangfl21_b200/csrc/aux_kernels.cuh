@@ -86,19 +86,23 @@ __global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned s
     }
 }
 
+// perm (nullable): internal id of each caller vertex id (locality relabeling, D15);
+// the output is written in caller order, coalesced, gathering from the internal array
 template <typename DistT>
 __global__ void finalize_kernel(const DistT* __restrict__ dist, unsigned long long* __restrict__ out, unsigned n,
-                                const unsigned long long* __restrict__ off, Ctl* ctl) {
+                                const unsigned long long* __restrict__ off, Ctl* ctl,
+                                const unsigned* __restrict__ perm = nullptr) {
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
     unsigned long long rv = 0, re = 0, mx = 0;
     for (unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
-        const DistT d = dist[v];
+        const unsigned long long iv = perm ? perm[v] : v;
+        const DistT d = dist[iv];
         if (d == DistInf<DistT>::value) {
             out[v] = ~0ull;
         } else {
             out[v] = (unsigned long long)d;
             rv += 1;
-            re += off[v + 1] - off[v];
+            re += off[iv + 1] - off[iv];
             mx = (unsigned long long)d > mx ? (unsigned long long)d : mx;
         }
     }
@@ -135,17 +139,19 @@ __global__ void interleave_f32_kernel(const unsigned* __restrict__ col, unsigned
 }
 
 __global__ void finalize_f32_kernel(const unsigned* __restrict__ dist, float* __restrict__ out, unsigned n,
-                                    const unsigned long long* __restrict__ off, Ctl* ctl) {
+                                    const unsigned long long* __restrict__ off, Ctl* ctl,
+                                    const unsigned* __restrict__ perm = nullptr) {
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
     unsigned long long rv = 0, re = 0, mx = 0;
     for (unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
-        const unsigned d = dist[v];
+        const unsigned long long iv = perm ? perm[v] : v;
+        const unsigned d = dist[iv];
         if (d >= 0x7F800000u) {  // never reached (internal sentinel) or +inf
             out[v] = __uint_as_float(0x7F800000u);
         } else {
             out[v] = __uint_as_float(d);
             rv += 1;
-            re += off[v + 1] - off[v];
+            re += off[iv + 1] - off[iv];
             mx = d > mx ? d : mx;
         }
     }
@@ -159,6 +165,50 @@ __global__ void finalize_f32_kernel(const unsigned* __restrict__ dist, float* __
         atomicAdd(&ctl->reach_v, rv);
         atomicAdd(&ctl->reach_e, re);
         atomicMax(&ctl->max_dist, mx);
+    }
+}
+
+// ---------------------------------------------------------------- locality relabeling (D15)
+// in-degree of every vertex (the number of arcs that gather/atomically update its dist)
+__global__ void indegree_kernel(const uint2* __restrict__ adj, unsigned long long m, unsigned* __restrict__ indeg) {
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long e = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; e < m; e += stride)
+        atomicAdd(&indeg[adj[e].x], 1u);
+}
+// sort keys: descending in-degree (ascending ~indeg), ties by id (stable sort of an iota)
+__global__ void relabel_keys_kernel(const unsigned* __restrict__ indeg, unsigned n, unsigned* __restrict__ key,
+                                    unsigned* __restrict__ iota) {
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
+        key[v] = ~indeg[v];
+        iota[v] = (unsigned)v;
+    }
+}
+// new_of_old[old_of_new[i]] = i; degree of internal vertex i
+__global__ void relabel_inverse_kernel(const unsigned* __restrict__ old_of_new, unsigned n,
+                                       const unsigned long long* __restrict__ off, unsigned* __restrict__ new_of_old,
+                                       unsigned long long* __restrict__ deg_new) {
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+        const unsigned o = old_of_new[i];
+        new_of_old[o] = (unsigned)i;
+        deg_new[i] = off[o + 1] - off[o];
+    }
+}
+// one warp per internal row: copy the old row's arcs, renaming their heads
+__global__ void relabel_arcs_kernel(const unsigned* __restrict__ old_of_new, const unsigned* __restrict__ new_of_old,
+                                    unsigned n, const unsigned long long* __restrict__ off,
+                                    const unsigned long long* __restrict__ off_new, const uint2* __restrict__ adj,
+                                    uint2* __restrict__ adj_new) {
+    const unsigned lane = threadIdx.x & 31;
+    const unsigned long long nw = (unsigned long long)gridDim.x * blockDim.x / 32;
+    for (unsigned long long i = ((unsigned long long)blockIdx.x * blockDim.x + threadIdx.x) / 32; i < n; i += nw) {
+        const unsigned o = old_of_new[i];
+        const unsigned long long b = off[o], e = off[o + 1], nb = off_new[i];
+        for (unsigned long long k = b + lane; k < e; k += 32) {
+            const uint2 a = adj[k];
+            adj_new[nb + (k - b)] = make_uint2(new_of_old[a.x], a.y);
+        }
     }
 }
 

@@ -2,6 +2,7 @@
 // workspace, launch sequence, status handling and retry.  All compute runs in
 // the kernels of adds_kernel.cuh / aux_kernels.cuh; there is no CPU fallback.
 #include <cuda_runtime.h>
+#include <cub/cub.cuh>
 
 #include <algorithm>
 #include <cmath>
@@ -112,6 +113,11 @@ struct sssp_graph {
     uint64_t m = 0;
     unsigned long long* d_off = nullptr;
     uint2* d_adj = nullptr;
+    // locality relabeling (D15): internal id of each caller id (device, for finalize;
+    // host, for the source); empty / nullptr = identity
+    unsigned* d_perm = nullptr;
+    std::vector<uint32_t> h_perm;
+    uint32_t max_indeg = 0;
     uint64_t sum_w = 0;
     uint32_t max_w = 0;
     uint32_t heur_k_span = 0;  // log2 initial Delta, max_w / B rule (ring span)
@@ -171,10 +177,11 @@ struct KVariant {
     void* fn;
     size_t smem;
 };
-template <typename DistT, int BT, bool kF = false, int EPT = 4, int MINB = 1024 / BT, bool PIPE = false, bool WLC = true>
+template <typename DistT, int BT, bool kF = false, int EPT = 4, int MINB = 1024 / BT, bool PIPE = false, bool WLC = true,
+          bool CA = false>
 KVariant kvar() {
     // (without the warp-local loop the per-warp continuation queues are not allocated)
-    return KVariant{(void*)adds_persistent_kernel<DistT, BT, EPT, MINB, PIPE, kF, WLC>,
+    return KVariant{(void*)adds_persistent_kernel<DistT, BT, EPT, MINB, PIPE, kF, WLC, CA>,
                     WLC ? Smem<DistT, BT, EPT>::bytes : Smem<DistT, BT, EPT>::o_wqv};
 }
 // SSSP_KVAR (experiments): 0 default (= 1 for 32-bit 512-thread CTAs); 1 pipelined 512x2/SM EPT 4; 2 pipelined 512x1/SM EPT 8;
@@ -195,6 +202,7 @@ KVariant persistent_variant(int bits, int bt, bool f32, bool wlc) {
         if (kv == 6) return kvar<uint32_t, 256, false, 8, 2, true>();
         if (bt == 128) return kvar<uint32_t, 128>();
         if (kv == 7) return kvar<uint32_t, 512>();  // 512 x 2/SM without the software pipeline (A/B)
+        if (kv == 11 && !wlc) return kvar<uint32_t, 512, false, 4, 2, true, false, true>();  // claim-ahead (A/B)
         if (bt == 512)  // default: pipelined; the warp-local loop only where it can run
             return wlc ? kvar<uint32_t, 512, false, 4, 2, true>() : kvar<uint32_t, 512, false, 4, 2, true, false>();
         if (bt == 1024) return kvar<uint32_t, 1024>();
@@ -458,6 +466,7 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
 
     const unsigned aux_grid = (unsigned)g->sm_count * 8 / conc + 1;
     CK(cudaEventRecord(w.ev[0], s), "event");
+    if (!g->h_perm.empty()) source = g->h_perm[source];  // internal id (D15)
     init_run_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, g->n, source, p.ctl, p.bk, p.ring, w.cap, h0,
                                                     p.expanded, p.filt);
     CK(cudaGetLastError(), "init kernel launch");
@@ -470,9 +479,11 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     }
     CK(cudaEventRecord(w.ev[2], s), "event");
     if constexpr (kF)
-        finalize_f32_kernel<<<aux_grid, 256, 0, s>>>((const unsigned*)p.dist, (float*)out_dev, g->n, g->d_off, p.ctl);
+        finalize_f32_kernel<<<aux_grid, 256, 0, s>>>((const unsigned*)p.dist, (float*)out_dev, g->n, g->d_off, p.ctl,
+                                                     g->d_perm);
     else
-        finalize_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, (unsigned long long*)out_dev, g->n, g->d_off, p.ctl);
+        finalize_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, (unsigned long long*)out_dev, g->n, g->d_off, p.ctl,
+                                                        g->d_perm);
     CK(cudaGetLastError(), "finalize kernel launch");
     CK(cudaEventRecord(w.ev[3], s), "event");
     CK(cudaMemcpyAsync(w.h_ctl, w.ctl.p, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "status copy");
@@ -524,13 +535,14 @@ sssp_status launch_nf(sssp_graph* g, Workspace& w, uint32_t source, void* out_de
     p.timeout_ns = (unsigned long long)(g->opts.timeout_ms ? g->opts.timeout_ms : 60000u) * 1000000ull;
     const unsigned aux_grid = (unsigned)g->sm_count * 8;
     CK(cudaEventRecord(w.ev[0], s), "event");
+    if (!g->h_perm.empty()) source = g->h_perm[source];  // internal id (D15)
     near_far_init_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, g->n, source, p.cnt, p.ctl, p.near[0]);
     CK(cudaGetLastError(), "init kernel launch");
     CK(cudaEventRecord(w.ev[1], s), "event");
     void* args[] = {(void*)&p};
     CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(256), args, 0, s), "Near-Far kernel launch");
     CK(cudaEventRecord(w.ev[2], s), "event");
-    finalize_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, out_dev, g->n, g->d_off, p.ctl);
+    finalize_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, out_dev, g->n, g->d_off, p.ctl, g->d_perm);
     CK(cudaGetLastError(), "finalize kernel launch");
     CK(cudaEventRecord(w.ev[3], s), "event");
     CK(cudaMemcpyAsync(w.h_ctl, w.ctl.p, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "status copy");
@@ -814,6 +826,98 @@ void sssp_options_default(sssp_options* o) {
 }  // extern "C"
 
 namespace {
+// Locality relabeling (D15): renumber vertices by descending in-degree so
+// the dist entries that most arcs gather from and atomically update share cache
+// lines (on a power-law graph the hot set becomes a few MB of L2-resident lines
+// instead of one hot entry per 32-byte sector).  The distance vector is a property
+// of the graph, not of its numbering: the source is mapped in, finalize gathers the
+// output back in caller order, so results are bit-identical.  Auto: on when the
+// in-degree is skewed (max > 64 x average); SSSP_FLAG_RELABEL / SSSP_FLAG_NO_RELABEL
+// force it; SSSP_RELABEL=0/1 in the environment overrides both (A/B).
+sssp_status relabel_graph(sssp_graph* g, const sssp_options& o) {
+    const unsigned n = g->n;
+    const unsigned long long m = g->m;
+    const unsigned aux_grid = (unsigned)g->sm_count * 8;
+    unsigned* indeg = nullptr;
+    CK(cudaMalloc(&indeg, (size_t)n * 4), "relabel: in-degrees");
+    cudaMemset(indeg, 0, (size_t)n * 4);
+    indegree_kernel<<<aux_grid, 256>>>(g->d_adj, m, indeg);
+    unsigned mx = 0;
+    {
+        unsigned* d_mx = nullptr;
+        void* tmp = nullptr;
+        size_t tb = 0;
+        cub::DeviceReduce::Max(tmp, tb, indeg, d_mx, n);
+        cudaMalloc(&d_mx, 4);
+        cudaMalloc(&tmp, tb);
+        cub::DeviceReduce::Max(tmp, tb, indeg, d_mx, n);
+        cudaError_t e = cudaMemcpy(&mx, d_mx, 4, cudaMemcpyDeviceToHost);
+        cudaFree(tmp);
+        cudaFree(d_mx);
+        if (e != cudaSuccess) {
+            cudaFree(indeg);
+            return cuda_fail(e, "relabel: max in-degree");
+        }
+    }
+    g->max_indeg = mx;
+    bool on = (double)mx > 64.0 * (double)m / (double)n;
+    if (o.flags & SSSP_FLAG_RELABEL) on = true;
+    if (o.flags & SSSP_FLAG_NO_RELABEL) on = false;
+    if (const char* e = std::getenv("SSSP_RELABEL")) on = std::atoi(e) != 0;
+    if (!on) {
+        cudaFree(indeg);
+        return SSSP_OK;
+    }
+    unsigned *key = nullptr, *key_out = nullptr, *iota = nullptr, *old_of_new = nullptr, *new_of_old = nullptr;
+    unsigned long long *deg_new = nullptr, *off_new = nullptr;
+    uint2* adj_new = nullptr;
+    void* tmp = nullptr;
+    size_t tb_sort = 0, tb_scan = 0;
+    auto cleanup = [&]() {
+        cudaFree(indeg); cudaFree(key); cudaFree(key_out); cudaFree(iota); cudaFree(old_of_new);
+        cudaFree(deg_new); cudaFree(tmp);
+    };
+    cudaError_t e = cudaSuccess;
+    if (e == cudaSuccess) e = cudaMalloc(&key, (size_t)n * 4);
+    if (e == cudaSuccess) e = cudaMalloc(&key_out, (size_t)n * 4);
+    if (e == cudaSuccess) e = cudaMalloc(&iota, (size_t)n * 4);
+    if (e == cudaSuccess) e = cudaMalloc(&old_of_new, (size_t)n * 4);
+    if (e == cudaSuccess) e = cudaMalloc(&new_of_old, (size_t)n * 4);
+    if (e == cudaSuccess) e = cudaMalloc(&deg_new, (size_t)(n + 1) * 8);
+    if (e == cudaSuccess) e = cudaMalloc(&off_new, (size_t)(n + 1) * 8);
+    if (e == cudaSuccess) e = cudaMalloc(&adj_new, (size_t)m * sizeof(uint2));
+    if (e == cudaSuccess) {
+        cub::DeviceRadixSort::SortPairs(nullptr, tb_sort, key, key_out, iota, old_of_new, (int)n);
+        cub::DeviceScan::ExclusiveSum(nullptr, tb_scan, deg_new, off_new, (int)n + 1);
+        e = cudaMalloc(&tmp, std::max(tb_sort, tb_scan));
+    }
+    if (e == cudaSuccess) {
+        relabel_keys_kernel<<<aux_grid, 256>>>(indeg, n, key, iota);
+        cub::DeviceRadixSort::SortPairs(tmp, tb_sort, key, key_out, iota, old_of_new, (int)n);
+        cudaMemset(deg_new + n, 0, 8);
+        relabel_inverse_kernel<<<aux_grid, 256>>>(old_of_new, n, g->d_off, new_of_old, deg_new);
+        cub::DeviceScan::ExclusiveSum(tmp, tb_scan, deg_new, off_new, (int)n + 1);
+        relabel_arcs_kernel<<<aux_grid, 256>>>(old_of_new, new_of_old, n, g->d_off, off_new, g->d_adj, adj_new);
+        e = cudaDeviceSynchronize();
+    }
+    if (e == cudaSuccess) {
+        g->h_perm.resize(n);
+        e = cudaMemcpy(g->h_perm.data(), new_of_old, (size_t)n * 4, cudaMemcpyDeviceToHost);
+    }
+    cleanup();
+    if (e != cudaSuccess) {
+        g->h_perm.clear();
+        cudaFree(new_of_old); cudaFree(off_new); cudaFree(adj_new);
+        return cuda_fail(e, "relabeling the graph");
+    }
+    cudaFree(g->d_off);
+    cudaFree(g->d_adj);
+    g->d_off = off_new;
+    g->d_adj = adj_new;
+    g->d_perm = new_of_old;
+    return SSSP_OK;
+}
+
 sssp_status create_impl(uint32_t n, uint64_t m, const uint64_t* row_offsets, const uint32_t* col, const uint32_t* w,
                         bool f32, const sssp_options* opts, sssp_graph** out) {
     if (!out) return fail(SSSP_ERR_INVALID_ARGUMENT, "out is NULL");
@@ -903,6 +1007,10 @@ sssp_status create_impl(uint32_t n, uint64_t m, const uint64_t* row_offsets, con
         return bail(fail(SSSP_ERR_INVALID_GRAPH, "w[" + std::to_string(scr[4]) + "] is negative or NaN"));
     g->sum_w = scr[2];
     g->max_w = (uint32_t)scr[3];
+    if (m) {
+        sssp_status rs = relabel_graph(g, o);
+        if (rs) return bail(rs);
+    }
     // initial Delta (reading R3): max_w / D (Meyer-Sanders' Theta(1/d) rule for Delta-stepping [15]),
     // or the Near-Far rule C * W / D with W = average weight, D = average degree, C = 32
     if (m && g->sum_w && !f32) {
@@ -942,6 +1050,7 @@ sssp_status sssp_graph_destroy(sssp_graph* g) {
     cudaDeviceSynchronize();
     if (g->d_off) cudaFree(g->d_off);
     if (g->d_adj) cudaFree(g->d_adj);
+    if (g->d_perm) cudaFree(g->d_perm);
     for (Workspace* w : g->ws) {
         w->release();
         delete w;
@@ -1054,6 +1163,13 @@ sssp_status sssp_graph_info(const sssp_graph* g, uint32_t* n, uint64_t* m, uint6
     if (sum_w) *sum_w = g->sum_w;
     if (max_w) *max_w = g->max_w;
     if (heuristic_delta_log2) *heuristic_delta_log2 = heuristic_k(g);
+    return SSSP_OK;
+}
+
+sssp_status sssp_graph_layout(const sssp_graph* g, uint32_t* relabeled, uint32_t* max_indeg) {
+    if (!g) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL graph");
+    if (relabeled) *relabeled = g->d_perm ? 1u : 0u;
+    if (max_indeg) *max_indeg = g->max_indeg;
     return SSSP_OK;
 }
 

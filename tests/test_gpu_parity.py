@@ -63,6 +63,26 @@ def test_golden_fixtures_warp_worker(name):
     assert st["worker"] == sssp.SSSP_WORKER_WARP
 
 
+@pytest.mark.parametrize("name", golden_names())
+def test_golden_fixtures_relabeled(name):
+    fx = load_golden(name)
+    g = gg.from_arcs(fx["n"], fx["arcs"])
+    d, st = gpu_dist(g, fx["source"], flags=sssp.SSSP_FLAG_RELABEL)
+    assert [int(x) for x in d] == fx["dist"]
+    assert st["reachable"] == fx["V"] and st["reach_edges"] == fx["E"]
+
+
+def test_relabel_auto_on_skewed_graphs_only():
+    # RMAT (power-law in-degrees) is relabeled, the grid is not; results identical either way
+    rmat = gg.make("rmat", scale_down=9)
+    s = int(gg.config_sources("rmat", rmat, 1)[0])
+    G = sssp.Graph.from_csr(rmat)
+    assert G.info()["relabeled"] == 1
+    assert np.array_equal(sssp.to_u64(G.run(s)), oracle.dijkstra(rmat, s)[0])
+    road = gg.make("road", scale_down=9)
+    assert sssp.Graph.from_csr(road).info()["relabeled"] == 0
+
+
 def test_worker_selection():
     # AUTO = the CTA worker (measured faster everywhere, D12); WARP on request
     rmat = gg.make("rmat", scale_down=10)
@@ -145,6 +165,10 @@ PERTURB = [
     dict(worker=sssp.SSSP_WORKER_WARP, delta_mode=1, delta_init=1),
     dict(worker=sssp.SSSP_WORKER_WARP, delta_mode=1, delta_init=1 << 30),
     dict(worker=sssp.SSSP_WORKER_WARP, flags=sssp.SSSP_FLAG_TRACE),
+    # locality relabeling (D15) forced on / off, with the 64-bit and Near-Far paths
+    dict(flags=sssp.SSSP_FLAG_RELABEL), dict(flags=sssp.SSSP_FLAG_NO_RELABEL),
+    dict(flags=sssp.SSSP_FLAG_RELABEL, dist_bits=64),
+    dict(flags=sssp.SSSP_FLAG_RELABEL, algorithm=sssp.SSSP_ALGO_NEAR_FAR),
 ]
 
 
