@@ -202,9 +202,12 @@ KVariant persistent_variant(int bits, int bt, bool f32, bool wlc) {
         if (kv == 6) return kvar<uint32_t, 256, false, 8, 2, true>();
         if (bt == 128) return kvar<uint32_t, 128>();
         if (kv == 7) return kvar<uint32_t, 512>();  // 512 x 2/SM without the software pipeline (A/B)
-        if (kv == 11 && !wlc) return kvar<uint32_t, 512, false, 4, 2, true, false, true>();  // claim-ahead (A/B)
-        if (bt == 512)  // default: pipelined; the warp-local loop only where it can run
-            return wlc ? kvar<uint32_t, 512, false, 4, 2, true>() : kvar<uint32_t, 512, false, 4, 2, true, false>();
+        if (bt == 512) {  // default: pipelined; the warp-local loop only where it can run, claim-ahead
+                          // elsewhere (SSSP_KVAR=11: without claim-ahead, A/B; sweeps §21)
+            if (wlc) return kvar<uint32_t, 512, false, 4, 2, true>();
+            return kv == 11 ? kvar<uint32_t, 512, false, 4, 2, true, false>()
+                            : kvar<uint32_t, 512, false, 4, 2, true, false, true>();
+        }
         if (bt == 1024) return kvar<uint32_t, 1024>();
         return kvar<uint32_t, 256>();
     }

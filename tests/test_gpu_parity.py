@@ -294,12 +294,32 @@ def test_full_size_config(config):
     s = int(gg.config_sources(config, g, 1)[0])
     ref, V, E = oracle.dijkstra(g, s)
     # the bench's launch configuration (auto worker) and each worker forced
-    for worker in (sssp.SSSP_WORKER_AUTO, sssp.SSSP_WORKER_CTA, sssp.SSSP_WORKER_WARP):
-        d, st = gpu_dist(g, s, worker=worker)
+    runs = [dict(worker=w) for w in (sssp.SSSP_WORKER_AUTO, sssp.SSSP_WORKER_CTA, sssp.SSSP_WORKER_WARP)]
+    runs += [dict(flags=sssp.SSSP_FLAG_NO_RELABEL if config == "rmat" else sssp.SSSP_FLAG_RELABEL)]
+    for opt in runs:
+        d, st = gpu_dist(g, s, **opt)
         bad = np.flatnonzero(d != ref)
-        assert bad.size == 0, f"worker={worker}: {bad.size} mismatches, first v={bad[:5]}"
+        assert bad.size == 0, f"{opt}: {bad.size} mismatches, first v={bad[:5]}"
         assert st["reachable"] == V and st["reach_edges"] == E
         assert st["dist_bits"] == 32
+
+
+def test_full_size_batch_sampled():
+    """Config 5 at full size in bench.py's launch configuration (RMAT-24, 4 sources in
+    flight): a seeded sample of the 512 batch sources, each row compared with the oracle,
+    plus the rank-partition the multi-GPU bench uses (sources[r::G])."""
+    g = gg.make("batch")
+    srcs = gg.sources(g, 512, gg.CONFIGS["batch"]["source_seed"])
+    rng = np.random.default_rng(5)
+    pick = np.sort(rng.choice(512, size=6, replace=False))
+    sample = srcs[pick]
+    G = sssp.Graph.from_csr(g, concurrent_sources=4)
+    D = G.run_batch(sample)
+    assert G.stats()["concurrency"] == 4
+    for i, s in enumerate(sample):
+        assert np.array_equal(sssp.to_u64(D[i]), oracle.dijkstra(g, int(s))[0]), f"source {int(s)}"
+    parts = [srcs[r::8] for r in range(8)]
+    assert sorted(np.concatenate(parts).tolist()) == sorted(srcs.tolist()) and len(set(srcs.tolist())) == 512
 
 
 def test_run_batch_distributed_single_rank():
