@@ -860,7 +860,12 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             // head-bucket children stay on chip: first in this warp's own queue (warp-local
             // continuation), then in the CTA's next batch (warp-aggregated slot grabs)
             unsigned wq_n = 0;  // warp-uniform fill of this warp's queue
+            unsigned wq_h = 0;  // logical index of its oldest entry (entries: [wq_h, wq_h + wq_n) mod kWQ)
             const unsigned wq0 = (unsigned)warp * kWQ;
+            // oldest first: an item that waited longest is the one most likely to hold the
+            // bucket open (FIFO vs LIFO on ROAD static 2^12: 34.4 vs 35.3 ms, sweeps §22);
+            // SSSP_EXP bit 18 selects newest first (A/B)
+            const bool wq_fifo = (p.exp & 0x40000u) == 0;
             // queue depth: past it children go to the CTA's next batch (shared by all
             // warps) or the ring (other CTAs); SSSP_EXP low byte overrides (A/B)
             const unsigned wqcap = (p.exp & 0xFFu) && (p.exp & 0xFFu) < kWQ ? (p.exp & 0xFFu) : kWQ;
@@ -873,15 +878,16 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     const unsigned wm = __ballot_sync(FULL, want);
                     if (wm) {
                         const unsigned pos = wq_n + __popc(wm & lt_mask);
+                        const unsigned ph = wq0 + (wq_h + pos) % kWQ;
                         if (want && pos < wqcap) {
                             if (!has_row) {
                                 rb = ld_stream_u64(p.off + v, pol_stream);
                                 rn = (unsigned)(ld_stream_u64(p.off + v + 1, pol_stream) - rb);
                             }
-                            s_wqv[wq0 + pos] = v;
-                            s_wqd[wq0 + pos] = (DistT)ndv;
-                            s_wqb[wq0 + pos] = rb;
-                            s_wqn[wq0 + pos] = rn;
+                            s_wqv[ph] = v;
+                            s_wqd[ph] = (DistT)ndv;
+                            s_wqb[ph] = rb;
+                            s_wqn[ph] = rn;
                             kept = true;
                         }
                         const unsigned nn = wq_n + __popc(wm);
@@ -1051,18 +1057,20 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             constexpr unsigned kWDeg = 8u * EPT;
             if constexpr (WLC) while (wq_n > 0) {
                 const unsigned take = wq_n < 32u ? wq_n : 32u;
-                const unsigned st0 = wq_n - take;
+                const unsigned st0 = wq_fifo ? wq_h : wq_h + wq_n - take;  // logical start of this hop's items
+                const unsigned ph = wq0 + (st0 + lane) % kWQ;
                 const bool has = lane < (int)take;
                 unsigned v = 0, deg = 0;
                 unsigned long long dv = kInf, b = 0;
                 if (has) {
-                    v = s_wqv[wq0 + st0 + lane];
-                    dv = (unsigned long long)s_wqd[wq0 + st0 + lane];
-                    b = s_wqb[wq0 + st0 + lane];
-                    deg = s_wqn[wq0 + st0 + lane];
+                    v = s_wqv[ph];
+                    dv = (unsigned long long)s_wqd[ph];
+                    b = s_wqb[ph];
+                    deg = s_wqn[ph];
                 }
                 __syncwarp();
-                wq_n = st0;
+                wq_n -= take;
+                if (wq_fifo) wq_h += take;
                 // long rows go back to the head bucket through the ring (their popper
                 // re-checks staleness)
                 const bool big = has && deg > kWDeg;
