@@ -130,6 +130,14 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
     if (head_switch && hsw < 255u) ++hsw;
     CtlDecision d{k, A, flo, steps | (hsw << 8), ceil, false, 0u};
     if (!p.dynamic) return d;
+    // the waste ceiling (hysteresis, below) holds for the rest of the run: letting it expire
+    // after 64 or 16 head switches regrew ROAD into wasteful Deltas (work 1.63x -> 2.0x,
+    // 43.9 -> 47 ms, sweeps §24).  SSSP_EXP bits 20..27 set an expiry count (A/B).
+    const unsigned ceil_life = (p.exp >> 20) & 0xFFu ? (p.exp >> 20) & 0xFFu : 255u;
+    if (ceil_life < 255u && hsw >= ceil_life) {
+        d.ceil = 0xffu;
+        ceil = 0xffu;
+    }
     const unsigned long long util = ((unsigned long long)(win > 0 ? win : 0) * p.avg_deg_x16) >> 4;
     const unsigned long long T = p.resident_threads;
     const bool low = util * 100ull < (unsigned long long)p.util_lo_pct * T;
