@@ -1093,20 +1093,21 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 for (int j = 0; j < EPT; ++j)
                     a[j] = lv && (unsigned)j < deg ? ld_stream_u2(p.adj + b + j, pol_stream) : make_uint2(0u, 0u);
                 lv = lv && cur >= dv;
-                bool fst = false;
+                // first-expansion bit for the controller: the atomicOr's result is consumed
+                // only after this hop's relaxations are issued (waiting for it here put a third
+                // dependent round trip into every hop of the dynamic mode)
+                unsigned fword = 0, fbit = 0;
                 if (lv && p.dynamic) {
-                    const unsigned bit = 1u << (v & 31);
-                    fst = (atomicOr(p.expanded + (v >> 5), bit) & bit) == 0;
+                    fbit = 1u << (v & 31);
+                    fword = atomicOr(p.expanded + (v >> 5), fbit);
                 }
                 if (!lv) deg = 0;
                 const unsigned nl = (unsigned)__popc(__ballot_sync(FULL, lv));
-                const unsigned nf = (unsigned)__popc(__ballot_sync(FULL, fst));
                 const unsigned ns = (unsigned)__popc(__ballot_sync(FULL, has && !lv && !big));
                 const unsigned sumdeg = __reduce_add_sync(FULL, deg);
                 const unsigned maxdeg = __reduce_max_sync(FULL, deg);
                 if (lane == 0) {
                     if (nl) atomicAdd(&s_wst[0], nl);
-                    if (nf) atomicAdd(&s_wst[1], nf);
                     if (sumdeg) atomicAdd(&s_wst[2], sumdeg);
                     if (ns) atomicAdd(&s_wst[3], ns);
                 }
@@ -1153,6 +1154,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         }
                     }
                 }
+                const unsigned nf = (unsigned)__popc(__ballot_sync(FULL, fbit != 0 && (fword & fbit) == 0));
+                if (lane == 0 && nf) atomicAdd(&s_wst[1], nf);
             }
         }
         if constexpr (CA) {

@@ -485,3 +485,26 @@ def test_filter16_resolution_change_keeps_results():
     for _ in range(2):
         d = sssp.to_u64(H.run(0))
         assert np.array_equal(d, oracle.dijkstra(ch, 0)[0])
+
+
+def test_bench_json_contract_small_config():
+    """bench.py's one-line JSON contract on the small config (the driver runs the same
+    code on configs[1]): required keys, device-timed value, e2e with host copies, clocks."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--config", "grid64", "--steps", "3",
+                          "--warmup", "3", "--e2e-steps", "2"], capture_output=True, text=True, timeout=600, cwd=root)
+    assert out.returncode == 0, out.stderr[-2000:]
+    line = json.loads(out.stdout.strip().splitlines()[-1])
+    for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
+              "vs_baseline", "dtype", "data", "config", "roofline", "cpu_baseline", "e2e", "gpu_launches", "clocks"):
+        assert k in line, k
+    assert line["value"] > 0 and line["steps"] == 3 and line["warmup"] == 3 and line["n_gpus"] == 1
+    assert line["gpu_launches"] >= 3 * 3
+    assert line["e2e"]["h2d_bytes_per_step"] > 0 and line["e2e"]["d2h_bytes_per_step"] > 0
+    assert line["roofline"]["peak"] > 0 and 0 < line["roofline"]["frac"] < 1
+    assert line["cpu_baseline"]["kind"] == "oracle" and line["cpu_baseline"]["cores"] == 1
+    assert "sm_mhz" in line["clocks"]
