@@ -60,7 +60,8 @@ def ncu_traffic(config):
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_summary.json")) as f:
             d = json.load(f)
-        return d.get(config, {}).get("dram_bytes_per_launch")
+        # a batch launch is one RMAT-24 source (on 1/c of the SMs): the rmat capture's bytes
+        return d.get("rmat" if config == "batch" else config, {}).get("dram_bytes_per_launch")
     except Exception:
         return None
 
