@@ -140,7 +140,9 @@ typedef struct sssp_options {
     uint32_t batch_min;        /* minimum items a CTA claims when enough are available; 0 = auto */
     uint32_t timeout_ms;       /* device watchdog (globaltimer); 0 = default 60000 */
     uint32_t trace_capacity;   /* trace ring entries when SSSP_FLAG_TRACE; 0 = 65536 */
-    uint32_t active_init;      /* initial number of active (claimable) buckets; 0 = auto (1) */
+    uint32_t active_init;      /* initial number of active (claimable) buckets; 0 = auto: 4 when
+                                  the average degree is > 8 (CTAs take the next bucket's items instead
+                                  of idling through the head bucket's tail), else 1 */
     uint32_t local_max;        /* head-bucket children a CTA keeps as its own next batch instead of
                                   publishing them, when its batch was at most half a CTA (latency regime);
                                   0 = auto = 128; see SSSP_FLAG_NO_LOCAL */

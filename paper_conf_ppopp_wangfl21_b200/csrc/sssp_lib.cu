@@ -450,7 +450,12 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     grid = std::max(1u, grid / conc);
     const unsigned k_max = kF ? 190u : (bits == 32 ? 31u : 63u);
     unsigned k = std::min(k0, k_max);
-    const unsigned A0 = g->opts.active_init ? g->opts.active_init : 1u;
+    // active buckets: auto = 4 on the throughput build (average degree > 8) -- CTAs
+    // that find the head bucket's published items exhausted take the next buckets' instead of
+    // idling through the head's tail (vs 1: RMAT -20 %, ER -17 %; vs 2: -1..4 %, sweeps §26) --
+    // and 1 on road-like graphs, where 2 gained only 2 % with more run-to-run spread and 3 sent
+    // the controller into a shrink spiral
+    const unsigned A0 = g->opts.active_init ? g->opts.active_init : (g->m > 8ull * g->n ? 4u : 1u);
     // initial floor of Delta (the controller never shrinks below it): the ring-span
     // value w_max / B, below which one maximum-weight hop from the head already
     // lands beyond the ring and is clipped ("the value of Delta should
