@@ -389,7 +389,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--algorithm", default="adds", choices=["adds", "nearfar"],
                     help="nearfar = the paper's BSP comparison system (ablation, NEXT-2)")
-    ap.add_argument("--concurrency", type=int, default=4, help="sources in flight per GPU for --config batch")
+    ap.add_argument("--concurrency", type=int, default=2,
+                    help="sources in flight per GPU for --config batch (measured 1/2/4/8: 44.9/46.6/44.3/25.7 GTEPS)")
     args = ap.parse_args()
     world, rank, local = dist_init()
     if args.impl == "reference":

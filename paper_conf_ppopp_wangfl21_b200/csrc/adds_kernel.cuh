@@ -70,7 +70,12 @@ struct Params {
     unsigned share_shift;      // a CTA claims about avail >> share_shift items
     unsigned local_max;        // head-bucket children a CTA keeps for itself (0 = off)
     unsigned warp_local;       // warp-local continuation in the latency regime (0 = off)
-    unsigned exp;              // experiment toggles (SSSP_EXP env, A/B on one box; 0 = production)
+    unsigned exp;              // experiment toggles (SSSP_EXP env, A/B on one box; 0 = production):
+                               //   bits 0-7   warp continuation queue depth cap (sweeps §19)
+                               //   bits 8-15  cumulative-ratio growth gate / 2, in % (§19)
+                               //   bit 16     publish overflowing head-bucket children at once (§19)
+                               //   bit 18     newest-first warp continuation queue (§22)
+                               //   bits 20-27 waste-ceiling lifetime in head switches (§24)
     unsigned short* filt;      // n x u16 upper bounds of dist in units of 2^filt_shift (nullptr = off)
     unsigned filt_shift;
     unsigned max_backoff_ns;
