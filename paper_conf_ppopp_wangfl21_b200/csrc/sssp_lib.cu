@@ -204,7 +204,11 @@ KVariant persistent_variant(int bits, int bt, bool f32, bool wlc) {
         if (kv == 7) return kvar<uint32_t, 512>();  // 512 x 2/SM without the software pipeline (A/B)
         if (bt == 512) {  // default: pipelined; the warp-local loop only where it can run, claim-ahead
                           // elsewhere (SSSP_KVAR=11: without claim-ahead, A/B; sweeps §21)
-            if (wlc) return kvar<uint32_t, 512, false, 4, 2, true>();
+            if (wlc) {  // warp-local build at 512x1/SM: 118 registers, no spills (at 2/SM: 64 registers,
+                        // 64 B stack); ROAD 41.6 -> 40.2 ms median of 6 pairs (sweeps §28). SSSP_KVAR=13: 2/SM (A/B)
+                if (kv == 13) return kvar<uint32_t, 512, false, 4, 2, true>();
+                return kvar<uint32_t, 512, false, 4, 1, true>();
+            }
             return kv == 11 ? kvar<uint32_t, 512, false, 4, 2, true, false>()
                             : kvar<uint32_t, 512, false, 4, 2, true, false, true>();
         }
