@@ -135,7 +135,7 @@ typedef struct sssp_options {
     uint64_t ring_items;       /* capacity of each bucket's circular array (items, rounded up to a
                                   power of two, >= 64); 0 = auto = max(2^16, next_pow2(n)) */
     uint32_t flags;            /* SSSP_FLAG_* */
-    uint32_t block_threads;    /* worker CTA size: 0 = auto (512), else 128/256/512/1024 */
+    uint32_t block_threads;    /* worker CTA size: 0 = auto (512; 128 on road-like graphs), else 128/256/512/1024 */
     uint32_t grid_ctas;        /* 0 = every co-resident CTA; else at most this many CTAs */
     uint32_t batch_min;        /* minimum items a CTA claims when enough are available; 0 = auto */
     uint32_t timeout_ms;       /* device watchdog (globaltimer); 0 = default 60000 */
@@ -146,7 +146,7 @@ typedef struct sssp_options {
     uint32_t local_max;        /* head-bucket children a CTA keeps as its own next batch instead of
                                   publishing them, when its batch was at most half a CTA (latency regime);
                                   0 = auto = 128; see SSSP_FLAG_NO_LOCAL */
-    uint32_t max_backoff_ns;   /* idle CTAs back off exponentially up to this (0 = auto = 2048) */
+    uint32_t max_backoff_ns;   /* idle CTAs back off exponentially up to this (0 = auto = 2048; 512 on road-like graphs) */
     uint32_t startup_permille; /* the controller may not grow Delta before this share of the vertices
                                   has been expanded or 32 head switches have happened (start-up
                                   frontiers are always small); default 20 (2%) */

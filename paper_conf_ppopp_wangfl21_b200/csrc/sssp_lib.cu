@@ -200,6 +200,9 @@ KVariant persistent_variant(int bits, int bt, bool f32, bool wlc) {
         if (kv == 4) return kvar<uint32_t, 512, false, 4, 1, true>();
         if (kv == 5) return kvar<uint32_t, 512, false, 8, 1, false>();
         if (kv == 6) return kvar<uint32_t, 256, false, 8, 2, true>();
+        // warp-local builds at smaller CTAs keep the same 128-register budget (no spills)
+        if (wlc && bt == 256 && kv != 13) return kvar<uint32_t, 256, false, 4, 2, true>();
+        if (wlc && bt == 128 && kv != 13) return kvar<uint32_t, 128, false, 4, 4, true>();
         if (bt == 128) return kvar<uint32_t, 128>();
         if (kv == 7) return kvar<uint32_t, 512>();  // 512 x 2/SM without the software pipeline (A/B)
         if (bt == 512) {  // default: pipelined; the warp-local loop only where it can run, claim-ahead
@@ -366,7 +369,7 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
     // one or two rounds of EPT arcs); on ER (degree 32) it serialised what the ring spreads
     // over CTAs (measured +13 %), so it is on by default only for average degree <= 8
     p.warp_local = warp_local_on(g) ? 1u : 0u;
-    p.max_backoff_ns = g->opts.max_backoff_ns ? g->opts.max_backoff_ns : 2048u;
+    p.max_backoff_ns = g->opts.max_backoff_ns ? g->opts.max_backoff_ns : (p.warp_local ? 512u : 2048u);  // §30
     p.prof = (g->opts.flags & SSSP_FLAG_PROFILE) ? 1u : 0u;
     p.expanded = (unsigned*)w.expanded.p;
     p.waste_lo = g->opts.waste_lo_permille;
@@ -439,7 +442,11 @@ unsigned heuristic_k(const sssp_graph* g) {
 template <typename DistT, bool kF>
 sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_dev, cudaStream_t s, int bits,
                        unsigned k0, unsigned conc) {
-    unsigned bt = g->opts.block_threads ? g->opts.block_threads : 512;
+    // auto CTA size: 512, except road-like graphs (warp-local build, 32-bit distances): four
+    // 128-thread CTAs per SM at the same 128-register budget -- more independent claimers on a
+    // latency-bound graph (ROAD 40.8 -> 38.0 ms with the 512 ns backoff cap, sweeps §30)
+    const bool wlc_auto = !kF && bits == 32 && warp_local_on(g);
+    unsigned bt = g->opts.block_threads ? g->opts.block_threads : (wlc_auto ? 128u : 512u);
     if (kF && bt != 256) bt = 512;  // float variants are built for 256/512-thread CTAs
     const bool warp_worker = use_warp_worker(g);
     if (warp_worker) bt = 512;
