@@ -1,6 +1,2 @@
-P="import sys,json
-for l in sys.stdin:
-    d=json.loads(l); print(d['opts'], d['kernel_ms'], d['work_E'])"
-for i in 1 2; do
-timeout 500 python tools/sweep.py --config road --sources 10 --sets '[{}, {"max_backoff_ns": 256}, {"max_backoff_ns": 128}, {"local_max": 64}, {"active_init": 2}]' 2>&1 | grep kernel_ms | python -c "$P"
-done
+timeout 300 python -c "import __graft_entry__ as g; g.smoke(); print('smoke ok')" 2>&1 | tail -1
+for i in 1 2; do timeout 300 python bench.py --steps 8 --warmup 3 --no-cpu-baseline 2>/dev/null | tail -1 | python -c "import sys,json;d=json.loads(sys.stdin.read());print(d['ms_per_step'],d['value'],d['e2e']['value'])"; done
