@@ -89,10 +89,11 @@ typedef enum sssp_status {
                                      (tools/l2_residency_bench.cu) it shrinks the normal L2 and LOWERS
                                      random-gather throughput (213 vs 263 G/s next to a 4 GB stream) */
 
-/* Worker granularity (options.worker) */
+/* Worker granularity (options.worker).  The warp-granular worker of round 1 was an
+ * ablation measured slower on every config (D12) and has been removed;
+ * the value 2 is rejected with SSSP_ERR_INVALID_ARGUMENT. */
 #define SSSP_WORKER_AUTO 0u
 #define SSSP_WORKER_CTA 1u
-#define SSSP_WORKER_WARP 2u
 
 /* Algorithms (options.algorithm) */
 #define SSSP_ALGO_ADDS 0u
@@ -162,11 +163,9 @@ typedef struct sssp_options {
                                   chunks that idle CTAs claim before bucket items (charged to the
                                   vertex's bucket, so the head cannot pass it early); 0 = auto
                                   (8 x CTA size), UINT32_MAX = off */
-    uint32_t worker;           /* unit of work of the ADDS persistent kernel: SSSP_WORKER_AUTO (0, = CTA),
+    uint32_t worker;           /* unit of work of the ADDS persistent kernel: SSSP_WORKER_AUTO (0) =
                                   SSSP_WORKER_CTA (a CTA claims up to a CTA-sized batch, expands it
-                                  cooperatively and keeps head-bucket children on chip) or
-                                  SSSP_WORKER_WARP (ablation: every warp is an independent worker with
-                                  up to 32 items and no CTA barrier; measured slower, D12) */
+                                  cooperatively and keeps head-bucket children on chip) */
     uint32_t reserved2[1];
 } sssp_options;
 
@@ -193,7 +192,7 @@ typedef struct sssp_stats {
     uint32_t status;             /* sssp_status of the last run (for SSSP_FLAG_ASYNC) */
     float batch_ms;              /* device time of the whole call on the caller's stream (CUDA events) */
     uint32_t concurrency;        /* sources that were in flight at once */
-    uint32_t worker;             /* SSSP_WORKER_CTA or SSSP_WORKER_WARP: the worker granularity that ran */
+    uint32_t worker;             /* SSSP_WORKER_CTA: the worker granularity that ran */
 } sssp_stats;
 
 /* One Delta-controller sample (written at each head-bucket switch and at each
@@ -291,6 +290,36 @@ sssp_status sssp_get_trace(sssp_graph *g, sssp_trace_entry *out, uint32_t cap, u
  * flushes, rounds, CTAs; then cycles in arc-window setup (owner scan + async
  * arc prefetch) and the window count.  *count receives min(cap, 16). */
 sssp_status sssp_get_profile(sssp_graph *g, uint64_t *out, uint32_t cap, uint32_t *count);
+
+/* Certificate of a distance vector (SURVEY.md §8(c) "What pins each part"): the
+ * O(n + m) checks that hold iff `dist` is the exact distance vector from `source`
+ * -- (i) dist[source] = 0; (ii) no arc (u, v, w) with dist[u] finite has
+ * dist[v] > dist[u] + w; (iii) every finite vertex is reachable from the source
+ * through tight arcs (dist[u] + w == dist[v]); (iv) unreachable entries carry the
+ * exact marker.  Float32-weight graphs use the IEEE round-to-nearest sum. */
+typedef struct sssp_certificate {
+    uint32_t exact;               /* 1 iff (i)-(iv) all hold */
+    uint32_t source_ok;           /* (i) */
+    uint64_t violated_arcs;       /* (ii): arcs whose head is above tail + weight */
+    uint64_t first_violated_tail; /* caller id of the smallest violated arc tail (UINT64_MAX: none) */
+    uint64_t unanchored;          /* (iii): finite vertices not reachable through tight arcs */
+    uint64_t first_unanchored;    /* caller id of the smallest such vertex (UINT64_MAX: none) */
+    uint64_t bad_markers;         /* (iv) float graphs: NaN / negative entries */
+    uint64_t reachable;           /* finite entries (V_dij when exact) */
+    uint64_t reach_edges;         /* sum of their out-degrees (E_dij when exact) */
+    uint32_t fixpoint_rounds;     /* rounds spent on tight arcs between equal distances (0-weight arcs) */
+    uint32_t reserved;
+} sssp_certificate;
+
+/* Checks `dist` (n entries in the caller's numbering: uint64 for integer graphs,
+ * float for float32-weight graphs; device memory on the graph's device or host
+ * memory) on the GPU with the certificate above: one pass over the arcs plus, only
+ * when tight zero-weight arcs exist, a fixed point over them.  Synchronous on
+ * `stream`; uses the handle's workspace as scratch, so not while a run is in flight
+ * (BUSY).  The verdict is in *out (SSSP_OK means the check ran, not that it passed).
+ * Errors: INVALID_ARGUMENT (NULL, source >= n), BUSY, DEVICE_MISMATCH, CUDA. */
+sssp_status sssp_certify(sssp_graph *g, uint32_t source, const void *dist, sssp_certificate *out,
+                         sssp_stream_t stream);
 
 /* Graph facts: n, m, sum of weights, max weight, and the heuristic initial
  * Delta (log2) under options.delta_heuristic: round(log2(max_w / B)),

@@ -70,12 +70,6 @@ struct Params {
     unsigned share_shift;      // a CTA claims about avail >> share_shift items
     unsigned local_max;        // head-bucket children a CTA keeps for itself (0 = off)
     unsigned warp_local;       // warp-local continuation in the latency regime (0 = off)
-    unsigned exp;              // experiment toggles (SSSP_EXP env, A/B on one box; 0 = production):
-                               //   bits 0-7   warp continuation queue depth cap (sweeps §19)
-                               //   bits 8-15  cumulative-ratio growth gate / 2, in % (§19)
-                               //   bit 16     publish overflowing head-bucket children at once (§19)
-                               //   bit 18     newest-first warp continuation queue (§22)
-                               //   bits 20-27 waste-ceiling lifetime in head switches (§24)
     unsigned short* filt;      // n x u16 upper bounds of dist in units of 2^filt_shift (nullptr = off)
     unsigned filt_shift;
     unsigned max_backoff_ns;
@@ -137,12 +131,7 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
     if (!p.dynamic) return d;
     // the waste ceiling (hysteresis, below) holds for the rest of the run: letting it expire
     // after 64 or 16 head switches regrew ROAD into wasteful Deltas (work 1.63x -> 2.0x,
-    // 43.9 -> 47 ms, sweeps §24).  SSSP_EXP bits 20..27 set an expiry count (A/B).
-    const unsigned ceil_life = (p.exp >> 20) & 0xFFu ? (p.exp >> 20) & 0xFFu : 255u;
-    if (ceil_life < 255u && hsw >= ceil_life) {
-        d.ceil = 0xffu;
-        ceil = 0xffu;
-    }
+    // 43.9 -> 47 ms, sweeps §24)
     const unsigned long long util = ((unsigned long long)(win > 0 ? win : 0) * p.avg_deg_x16) >> 4;
     const unsigned long long T = p.resident_threads;
     const bool low = util * 100ull < (unsigned long long)p.util_lo_pct * T;
@@ -159,7 +148,7 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
     // cumulative-ratio gate on growth: 2.5x Dijkstra's vertex work (road-like graphs sit
     // at 1.6-1.7x at their time-optimal Delta; a 1.5x gate pinned them one step below it,
     // profiles/r01_sweeps.md §19)
-    const unsigned ratio_gate = (p.exp >> 8) & 0xFFu ? ((p.exp >> 8) & 0xFFu) * 2u : 250u;  // SSSP_EXP A/B
+    constexpr unsigned ratio_gate = 250u;
     const bool frugal = (!waste_known || waste < p.waste_lo) &&
                         (ratio_x100 < ratio_gate || !waste_known || waste * 2 < p.waste_lo) && progressed;
     const bool clipping = (total >= 64 && tail * 100 >= (long long)p.clip_pct * total) || (clip_known && clip >= 500);
@@ -318,6 +307,7 @@ __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lan
                                      ld_relaxed_u32(&p.ctl->head_switches) >= 32u);
     const Head nhd{rehead(hd.h + o, k, d.k),
                    pack_meta((hs + o) & (nb - 1), d.k, d.A, d.flo, d.since, d.ceil)};
+    SSSP_FUZZ_AT(FZ_HEAD);
     commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 1u, d.flags);
     return false;
 }
@@ -433,6 +423,7 @@ __device__ unsigned claim_batch(const Params<DistT>& p, int lane, unsigned& o_sl
             unsigned long long* avp = &p.bk[kSplitQ].avail.v;
             const long long old = (long long)atomicAdd(avp, (unsigned long long)(-1ll));
             if (old > 0) {
+                SSSP_FUZZ_AT(FZ_CLAIM);
                 ix = atomicAdd(&p.bk[kSplitQ].claim.v, 1ull);
                 got = 1;
             } else {
@@ -460,7 +451,10 @@ __device__ unsigned claim_batch(const Params<DistT>& p, int lane, unsigned& o_sl
             const long long old = (long long)atomicAdd(avp, (unsigned long long)(-want));
             const long long g = old <= 0 ? 0 : (old < want ? old : want);
             if (g < want) atomicAdd(avp, (unsigned long long)(want - g));
-            if (g > 0) ix = atomicAdd(&p.bk[sl].claim.v, (unsigned long long)g);
+            if (g > 0) {
+                SSSP_FUZZ_AT(FZ_CLAIM);
+                ix = atomicAdd(&p.bk[sl].claim.v, (unsigned long long)g);
+            }
             g32 = (unsigned)g;
             sl32 = sl;
         }
@@ -487,6 +481,7 @@ __device__ unsigned spawn_chunks(const Params<DistT>& p, unsigned v, unsigned lo
     const unsigned extra = (deg - 1) / S;
     atomicAdd(&p.bk[slot].local.v, (unsigned long long)extra);
     const unsigned long long t0 = atomicAdd(&p.bk[kSplitQ].reserve.v, (unsigned long long)extra);
+    SSSP_FUZZ_AT(FZ_CHUNK);
     if (t0 + extra > p.tcap && t0 + extra - p.tcap > ld_relaxed_u64(&p.bk[kSplitQ].claim.v)) {
         atomicOr(&p.ctl->status, kStRingOverflow);  // would lap an unclaimed chunk: regrow and re-run
         return S;
@@ -505,6 +500,7 @@ __device__ unsigned spawn_chunks(const Params<DistT>& p, unsigned v, unsigned lo
         tp->slot = slot;
     }
     __threadfence();  // payloads before their len markers
+    SSSP_FUZZ_AT(FZ_CHUNK);
     for (unsigned c = 1; c <= extra; ++c) {
         const unsigned rest = deg - c * S;
         st_relaxed_u32(&p.tasks[(t0 + c - 1) & (p.tcap - 1)].len, rest < S ? rest : S);
@@ -696,7 +692,6 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         // warp-local continuation (same regime): a warp runs its own head-bucket
         // children hop after hop with no CTA barrier (D9)
         const bool wlc = WLC && lcap != 0 && p.warp_local != 0;
-        const bool direct_head = wlc && (p.exp & 0x10000u) != 0;  // A/B (SSSP_EXP bit 16)
 
         // ------------------------------------------------------------ pop + stale check
         const Head hd = s_head;
@@ -739,6 +734,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     const unsigned long long idx = (s_idx + tid) & (p.cap - 1);
                     char* sp = p.ring + ((size_t)slot * p.cap + idx) * IT::kBytes;
                     unsigned spins = 0;
+                    SSSP_FUZZ_AT(FZ_POP);
                     while (!(loaded = IT::load(sp, v, d))) {  // reserved, store not landed yet
                         if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;  // aborted run
                     }
@@ -877,11 +873,9 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             const unsigned wq0 = (unsigned)warp * kWQ;
             // oldest first: an item that waited longest is the one most likely to hold the
             // bucket open (FIFO vs LIFO on ROAD static 2^12: 34.4 vs 35.3 ms, sweeps §22);
-            // SSSP_EXP bit 18 selects newest first (A/B)
-            const bool wq_fifo = (p.exp & 0x40000u) == 0;
-            // queue depth: past it children go to the CTA's next batch (shared by all
-            // warps) or the ring (other CTAs); SSSP_EXP low byte overrides (A/B)
-            const unsigned wqcap = (p.exp & 0xFFu) && (p.exp & 0xFFu) < kWQ ? (p.exp & 0xFFu) : kWQ;
+            // past the queue depth children go to the CTA's next batch (shared by all warps)
+            // or the ring (other CTAs)
+            constexpr unsigned wqcap = kWQ;
             // rb/rn: the child's row (begin, degree) when already fetched (has_row), else it
             // is loaded here
             auto keep = [&](const bool want, const unsigned v, const unsigned long long ndv, const bool has_row,
@@ -908,7 +902,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         wq_n = nn < wqcap ? nn : wqcap;
                     }
                 }
-                if (lcap && !direct_head) {  // (direct_head: overflow goes to the ring at once)
+                if (lcap) {
                     const bool w2 = want && !kept;
                     const unsigned lm = __ballot_sync(FULL, w2);
                     if (lm) {
@@ -927,22 +921,16 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             };
             // everything else: warp-aggregated staging for the CTA flush at batch end
             // (or direct publication when the staging area is full)
-            // direct (warp-uniform): publish now instead of at batch end -- head-bucket
-            // children that overflow the on-chip queues in the latency regime, which idle
-            // CTAs should get while this CTA is still running its chains
-            auto emit = [&](const bool pg, const unsigned v, const unsigned long long ndv, const unsigned o,
-                            const bool direct = false) {
+            auto emit = [&](const bool pg, const unsigned v, const unsigned long long ndv, const unsigned o) {
                 const unsigned act = __ballot_sync(FULL, pg);
                 if (!act) return;
                 // warp-aggregated staging slot for the CTA flush at batch end
                 const int leader = __ffs(act) - 1;
                 const unsigned nact = (unsigned)__popc(act);
                 unsigned pos = 0;
-                if (!direct) {
-                    if (lane == leader) pos = atomicAdd(&s_total, nact);
-                    pos = __shfl_sync(FULL, pos, leader);
-                }
-                if (!direct && pos + nact <= (unsigned)kStage) {
+                if (lane == leader) pos = atomicAdd(&s_total, nact);
+                pos = __shfl_sync(FULL, pos, leader);
+                if (pos + nact <= (unsigned)kStage) {
                     if (pg) {
                         const unsigned peers = __match_any_sync(act, o);
                         const int pl = __ffs(peers) - 1;
@@ -959,7 +947,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     // publish directly -- one reserve/avail pair per (warp, bucket)
                     if (pg) {
                         const unsigned my = pos + __popc(act & lt_mask);
-                        if (!direct && my < (unsigned)kStage) s_soff[my] = 0xFF;
+                        if (my < (unsigned)kStage) s_soff[my] = 0xFF;
                         const unsigned peers = __match_any_sync(act, o);
                         const int pl = __ffs(peers) - 1;
                         const unsigned sl = (hs + o) & nbm;
@@ -969,11 +957,13 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                             b0 = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
                             if (b0 + c > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
                             atomicAdd(&s_direct, c);
+                            SSSP_FUZZ_AT(FZ_RESERVE);
                         }
                         b0 = __shfl_sync(peers, b0, pl);
                         const unsigned long long idx = b0 + __popc(peers & lt_mask);
                         // the slot's one writer this run (D13); beyond cap the run is aborted
                         if (idx < p.cap) IT::store(p.ring + ((size_t)sl * p.cap + idx) * IT::kBytes, IT::make(v, ndv));
+                        SSSP_FUZZ_AT(FZ_PUBLISH);
                         __syncwarp(peers);
                         if (lane == pl) atomicAdd(&p.bk[sl].avail.v, (unsigned long long)__popc(peers));
                     }
@@ -1022,12 +1012,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     if (!__any_sync(FULL, push[j])) continue;
                     const unsigned o = push[j] ? bucket_of<kF>(nd[j], k, hd.h, p.nb) : 0u;
                     const bool kept = keep(push[j] && o == 0, a[j].x, nd[j], false, 0ull, 0u);
-                    if (direct_head) {
-                        emit(push[j] && !kept && o != 0, a[j].x, nd[j], o);
-                        emit(push[j] && !kept && o == 0, a[j].x, nd[j], 0u, true);
-                    } else {
-                        emit(push[j] && !kept, a[j].x, nd[j], o);
-                    }
+                    emit(push[j] && !kept, a[j].x, nd[j], o);
                 }
             };
             if (PIPE && we > wb + kChunk) {
@@ -1070,7 +1055,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             constexpr unsigned kWDeg = 8u * EPT;
             if constexpr (WLC) while (wq_n > 0) {
                 const unsigned take = wq_n < 32u ? wq_n : 32u;
-                const unsigned st0 = wq_fifo ? wq_h : wq_h + wq_n - take;  // logical start of this hop's items
+                const unsigned st0 = wq_h;  // logical start of this hop's items
                 const unsigned ph = wq0 + (st0 + lane) % kWQ;
                 const bool has = lane < (int)take;
                 unsigned v = 0, deg = 0;
@@ -1083,11 +1068,11 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
                 __syncwarp();
                 wq_n -= take;
-                if (wq_fifo) wq_h += take;
+                wq_h += take;
                 // long rows go back to the head bucket through the ring (their popper
                 // re-checks staleness)
                 const bool big = has && deg > kWDeg;
-                emit(big, v, dv, 0u, direct_head);
+                emit(big, v, dv, 0u);
                 bool lv = has && !big;
                 // the stale re-check is in flight together with the first arc loads (one
                 // round trip); skipping it expands superseded children (measured 1.7x ->
@@ -1151,12 +1136,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         if (!__any_sync(FULL, push[j])) continue;
                         const unsigned o = push[j] ? bucket_of<kF>(nd[j], k, hd.h, p.nb) : 0u;
                         const bool kept = keep(push[j] && o == 0, a[j].x, nd[j], true, rb[j], (unsigned)(re[j] - rb[j]));
-                        if (direct_head) {
-                            emit(push[j] && !kept && o != 0, a[j].x, nd[j], o);
-                            emit(push[j] && !kept && o == 0, a[j].x, nd[j], 0u, true);
-                        } else {
-                            emit(push[j] && !kept, a[j].x, nd[j], o);
-                        }
+                        emit(push[j] && !kept, a[j].x, nd[j], o);
                     }
                 }
                 const unsigned nf = (unsigned)__popc(__ballot_sync(FULL, fbit != 0 && (fword & fbit) == 0));
@@ -1200,6 +1180,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         // returning atomic: the reserve (which also counts the children for
                         // termination) is performed before this CTA's completion atomic
                         const unsigned long long b = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
+                        SSSP_FUZZ_AT(FZ_RESERVE);
                         s_base[lane] = b;
                         if (b + c > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
                     }
@@ -1210,6 +1191,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     if (o == 0xFF) continue;  // hole left by a direct publication
                     const unsigned sl = (hs + o) & nbm;
                     const unsigned long long idx = s_base[o] + s_rank[i];
+                    SSSP_FUZZ_AT(FZ_PUBLISH);
                     // the slot's one writer this run (D13); beyond cap the run is aborted
                     if (idx < p.cap) IT::store(p.ring + ((size_t)sl * p.cap + idx) * IT::kBytes, s_items[i]);
                 }
@@ -1259,8 +1241,11 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 c_local += s_wst[4];
                 s_wst[0] = s_wst[1] = s_wst[2] = s_wst[3] = s_wst[4] = 0;
             }
-            // one atomic: the kept children inherit the parents' accounting
-            if (got > kept) atomicAdd(&p.bk[slot].done.v, (unsigned long long)(got - kept));
+            // one atomic: the kept children inherit the parents' accounting; a completion
+            // is a release (common.cuh red_release_add_u64): the children's reserve
+            // atomics above are ordered before it by the CTA barrier
+            SSSP_FUZZ_AT(FZ_COMPLETE);
+            if (got > kept) red_release_add_u64(&p.bk[slot].done.v, (unsigned long long)(got - kept));
             else if (kept > got) atomicAdd(&p.bk[slot].local.v, (unsigned long long)(kept - got));
             c_push += kept;
             c_local += kept;

@@ -245,6 +245,40 @@ __device__ __forceinline__ unsigned long long globaltimer() {
     return t;
 }
 
+// Completion counter update with gpu-scope release semantics: every write of the
+// CTA that precedes it (children's reserve atomics and ring stores, ordered by the
+// CTA barrier) is visible to whoever acquire-reads the counter and sees the
+// increment (try_advance / bucket_pending read `done` with ld.acquire before
+// `reserve` and `local`), so a bucket can never look complete while one of its
+// items' children is not yet counted (exact termination).
+__device__ __forceinline__ void red_release_add_u64(unsigned long long* p, unsigned long long v) {
+    asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// ---- schedule fuzzing (libsssp_fuzz.so, built with -DSSSP_FUZZ; tests only).
+// A hash of the SM clock, the global timer, the CTA, the thread and the site picks
+// one call in four and sleeps 32 ns .. 4 us there, so the worklist protocol is
+// exercised under reorderings the natural schedule rarely produces: a reserved
+// slot published late, a claim separated from its read_ptr update, a completion
+// or a head advance delayed past other CTAs' work.
+enum FuzzSite : unsigned { FZ_CLAIM = 1, FZ_POP, FZ_RESERVE, FZ_PUBLISH, FZ_COMPLETE, FZ_HEAD, FZ_CHUNK };
+#ifdef SSSP_FUZZ
+__device__ __forceinline__ void fuzz_delay(unsigned site) {
+    const unsigned long long t = globaltimer() ^ ((unsigned long long)clock64() << 7);
+    unsigned h = (unsigned)(t ^ (t >> 32)) * 0x9E3779B1u;
+    h ^= blockIdx.x * 0x85EBCA6Bu ^ threadIdx.x * 0xC2B2AE35u ^ site * 0x27D4EB2Fu;
+    h ^= h >> 15;
+    h *= 0x2C1B3C6Du;
+    h ^= h >> 12;
+    h *= 0x297A2D39u;
+    h ^= h >> 15;
+    if ((h & 3u) == 0u) __nanosleep(32u + ((h >> 4) & 4095u));
+}
+#define SSSP_FUZZ_AT(site) ::adds::fuzz_delay(site)
+#else
+#define SSSP_FUZZ_AT(site) ((void)0)
+#endif
+
 // 128-bit CAS on the head state (sm_90+: atom.cas.b128).
 __device__ __forceinline__ bool cas_head(Head* addr, Head expect, Head desired, Head& seen) {
     unsigned long long o0, o1;

@@ -10,12 +10,13 @@
 #include <cstring>
 #include <cstdlib>
 #include <string>
+#include <type_traits>
 #include <vector>
 
 #include "../../include/sssp.h"
 #include "adds_kernel.cuh"
-#include "adds_warp_kernel.cuh"
 #include "aux_kernels.cuh"
+#include "certify_kernels.cuh"
 #include "nearfar_kernel.cuh"
 #include "bucket_map.h"
 
@@ -127,11 +128,13 @@ struct sssp_graph {
     sssp_options opts{};
     int sm_count = 0;
     std::vector<Workspace*> ws;
-    DevBuf scratch, hostout;
+    DevBuf scratch, hostout, cert;
     cudaEvent_t bev[2] = {nullptr, nullptr};  // batch start / end on the caller's stream
     int cur_bits = 32;       // 64 after a 32-bit overflow was observed (sticky)
     unsigned filt_shift_hint = 0;  // 1 + filter resolution fitted to the last run's max distance
     size_t persist_max = 0;  // device's L2 persisting set-aside limit (bytes)
+    bool persist_saved = false;  // SSSP_FLAG_L2_PERSIST raised the device limit: restore after the run
+    size_t persist_prev = 0;
     bool busy = false;
     bool async_pending = false;
     sssp_stats stats{};
@@ -165,7 +168,9 @@ sssp_status check_options(const sssp_options& o) {
     if (o.waste_lo_permille > 1000 || o.waste_hi_permille > 1000) return fail(SSSP_ERR_INVALID_ARGUMENT, "waste permille");
     if (o.concurrent_sources > 64) return fail(SSSP_ERR_INVALID_ARGUMENT, "concurrent_sources > 64");
     if (o.algorithm > SSSP_ALGO_NEAR_FAR) return fail(SSSP_ERR_INVALID_ARGUMENT, "algorithm");
-    if (o.worker > SSSP_WORKER_WARP) return fail(SSSP_ERR_INVALID_ARGUMENT, "worker");
+    if (o.worker > SSSP_WORKER_CTA)
+        return fail(SSSP_ERR_INVALID_ARGUMENT, "worker: only SSSP_WORKER_AUTO / SSSP_WORKER_CTA (the warp-granular "
+                                               "ablation was measured slower everywhere and removed, DESIGN.md D12)");
     return SSSP_OK;
 }
 
@@ -184,37 +189,20 @@ KVariant kvar() {
     return KVariant{(void*)adds_persistent_kernel<DistT, BT, EPT, MINB, PIPE, kF, WLC, CA>,
                     WLC ? Smem<DistT, BT, EPT>::bytes : Smem<DistT, BT, EPT>::o_wqv};
 }
-// SSSP_KVAR (experiments): 0 default (= 1 for 32-bit 512-thread CTAs); 1 pipelined 512x2/SM EPT 4; 2 pipelined 512x1/SM EPT 8;
-// (3, pipelined 1024x1/SM, removed: it hit the watchdog on ROAD, unexplained); 4 pipelined 512x1/SM EPT 4; 5 plain 512x1/SM EPT 8;
-// 6 pipelined 256x2/SM EPT 8; 7 plain 512x2/SM EPT 4 (the pre-pipeline default)
-static int kvar_env() {
-    const char* e = std::getenv("SSSP_KVAR");
-    return e ? std::atoi(e) : 0;
-}
+// The kernel instantiation for a launch shape (each variant's BT is the CTA size it
+// is launched with).  32-bit distances: road-like graphs (warp-local build) run
+// 128-thread CTAs x 4/SM at 128 registers (ROAD 40.8 -> 38.0 ms, sweeps §30) or
+// 512 x 1/SM when asked; the throughput build is pipelined with claim-ahead at
+// 512 x 2/SM (sweeps §8, §21).  64-bit distances and float32 weights use the plain
+// build at the requested CTA size.
 KVariant persistent_variant(int bits, int bt, bool f32, bool wlc) {
     if (f32) return bt == 256 ? kvar<uint32_t, 256, true>() : kvar<uint32_t, 512, true>();
-    const int kv = kvar_env();
     if (bits == 32) {
-        if (kv == 1) return kvar<uint32_t, 512, false, 4, 2, true>();
-        if (kv == 2) return kvar<uint32_t, 512, false, 8, 1, true>();
-        if (kv == 4) return kvar<uint32_t, 512, false, 4, 1, true>();
-        if (kv == 5) return kvar<uint32_t, 512, false, 8, 1, false>();
-        if (kv == 6) return kvar<uint32_t, 256, false, 8, 2, true>();
-        // warp-local builds at smaller CTAs keep the same 128-register budget (no spills)
-        if (wlc && bt == 256 && kv != 13) return kvar<uint32_t, 256, false, 4, 2, true>();
-        if (wlc && bt == 128 && kv != 13) return kvar<uint32_t, 128, false, 4, 4, true>();
+        if (wlc && bt == 128) return kvar<uint32_t, 128, false, 4, 4, true>();
+        if (wlc && bt == 256) return kvar<uint32_t, 256, false, 4, 2, true>();
+        if (wlc && bt == 512) return kvar<uint32_t, 512, false, 4, 1, true>();
         if (bt == 128) return kvar<uint32_t, 128>();
-        if (kv == 7) return kvar<uint32_t, 512>();  // 512 x 2/SM without the software pipeline (A/B)
-        if (bt == 512) {  // default: pipelined; the warp-local loop only where it can run, claim-ahead
-                          // elsewhere (SSSP_KVAR=11: without claim-ahead, A/B; sweeps §21)
-            if (wlc) {  // warp-local build at 512x1/SM: 118 registers, no spills (at 2/SM: 64 registers,
-                        // 64 B stack); ROAD 41.6 -> 40.2 ms median of 6 pairs (sweeps §28). SSSP_KVAR=13: 2/SM (A/B)
-                if (kv == 13) return kvar<uint32_t, 512, false, 4, 2, true>();
-                return kvar<uint32_t, 512, false, 4, 1, true>();
-            }
-            return kv == 11 ? kvar<uint32_t, 512, false, 4, 2, true, false>()
-                            : kvar<uint32_t, 512, false, 4, 2, true, false, true>();
-        }
+        if (bt == 512) return kvar<uint32_t, 512, false, 4, 2, true, false, true>();
         if (bt == 1024) return kvar<uint32_t, 1024>();
         return kvar<uint32_t, 256>();
     }
@@ -222,28 +210,6 @@ KVariant persistent_variant(int bits, int bt, bool f32, bool wlc) {
     if (bt == 512) return kvar<unsigned long long, 512>();
     if (bt == 1024) return kvar<unsigned long long, 1024>();
     return kvar<unsigned long long, 256>();
-}
-
-// Warp-granular worker (adds_warp_kernel.cuh): 512-thread CTAs, 2 per SM, EPT 4.
-template <typename DistT, bool kF = false>
-KVariant wvar() {
-    return KVariant{(void*)adds_warp_kernel<DistT, 512, 4, 2, kF>, (512 / 32) * sizeof(WarpSmem<DistT>)};
-}
-KVariant warp_variant(int bits, bool f32) {
-    if (f32) return wvar<uint32_t, true>();
-    return bits == 32 ? wvar<uint32_t>() : wvar<unsigned long long>();
-}
-// Which worker runs (D12).  The warp worker (no CTA barriers) was the
-// hypothesis for the throughput regime; measured on B200 it is slower on every
-// config (ER 16.3 vs 11.8 ms, RMAT 7.6 vs 6.7, ROAD 130 vs 44: 16x more claimers
-// on the same bucket counters, and per-warp batches of 32 items pay the claim
-// round trips 16x as often), so AUTO = CTA and the warp worker is an ablation.
-// SSSP_KVAR=8 / 9 force warp / CTA (A/B on one box).
-bool use_warp_worker(const sssp_graph* g) {
-    const char* e = std::getenv("SSSP_KVAR");
-    if (e && std::atoi(e) == 8) return true;
-    if (e && std::atoi(e) == 9) return false;
-    return g->opts.worker == SSSP_WORKER_WARP;
 }
 
 // warp-local continuation (D10): on for road-like graphs (average degree <= 8) unless disabled
@@ -273,7 +239,7 @@ unsigned split_degree(const sssp_graph* g, unsigned bt) {
     if (g->opts.split_degree == 0xFFFFFFFFu) return 0u;
     // (chunk lengths must stay below the queue's slot-state markers, common.cuh)
     if (g->opts.split_degree) return std::min(g->opts.split_degree, 1u << 31);
-    return 8u * bt;  // warp worker: bt = 128 -> 1024 arcs
+    return 8u * bt;
 }
 
 // Hub-split chunk queue: enough entries for every arc of the graph in chunks of
@@ -379,18 +345,18 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
     // L2 residency of dist (D5): reserve the persisting set-aside for
     // the concurrently live dist arrays and mark dist accesses evict_last over
     // the fraction that fits
+    // The device-wide set-aside is touched only when the caller opts in; the previous
+    // limit is restored when the run ends (restore_persist).
     p.keep_frac = 0.0f;
-    if (!(g->opts.flags & SSSP_FLAG_L2_PERSIST) && g->persist_max) {
-        // the driver's default set-aside (~25 MB on B200) only shrinks the normal L2
-        size_t cur = 0;
-        cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
-        if (cur) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
-    }
     if ((g->opts.flags & SSSP_FLAG_L2_PERSIST) && g->persist_max) {
         const size_t want = (size_t)g->n * sizeof(DistT) * conc;
         const size_t use = std::min(want, g->persist_max);
         size_t cur = 0;
         cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+        if (!g->persist_saved) {
+            g->persist_saved = true;
+            g->persist_prev = cur;
+        }
         if (cur < use) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, use);
         cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
         p.keep_frac = want ? (float)std::min(1.0, (double)std::min(cur, use) / (double)want) : 0.0f;
@@ -405,10 +371,6 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
         // first run on a graph: 2^s = max_w / 16; afterwards the resolution that maps the
         // previous run's largest distance below 60000 (the result never depends on it)
         p.filt_shift = g->filt_shift_hint ? g->filt_shift_hint - 1 : (lg > 4 ? lg - 4 : 0);
-    }
-    {
-        const char* e = std::getenv("SSSP_EXP");
-        p.exp = e ? (unsigned)std::strtoul(e, nullptr, 0) : 0u;
     }
     p.tasks = (SplitTask*)w.tasks.p;
     p.tcap = w.tcap;
@@ -448,9 +410,7 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     const bool wlc_auto = !kF && bits == 32 && warp_local_on(g);
     unsigned bt = g->opts.block_threads ? g->opts.block_threads : (wlc_auto ? 128u : 512u);
     if (kF && bt != 256) bt = 512;  // float variants are built for 256/512-thread CTAs
-    const bool warp_worker = use_warp_worker(g);
-    if (warp_worker) bt = 512;
-    const KVariant kv = warp_worker ? warp_variant(bits, kF) : persistent_variant(bits, (int)bt, kF, warp_local_on(g));
+    const KVariant kv = persistent_variant(bits, (int)bt, kF, warp_local_on(g));
     void* fn = kv.fn;
     CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kv.smem), "smem attribute");
     int occ = 0;
@@ -474,14 +434,6 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     const unsigned span = kF ? heuristic_k(g) : g->heur_k_span;
     Head h0{0ull, pack_meta(0, k, A0, std::min(k, span), 0)};
     Params<DistT> p = make_params<DistT>(g, w, grid, bt, k_max, conc);
-    if (warp_worker) {
-        // a warp claims up to 32 items; split hubs into 8 rounds of 32 x EPT arcs
-        unsigned sh = 0;
-        while ((1u << (sh + 1)) <= grid * (bt / 32)) ++sh;
-        p.share_shift = sh > 2 ? sh - 2 : 0;
-        p.split_deg = split_degree(g, 128);
-        p.prof = 0;
-    }
 
     const unsigned aux_grid = (unsigned)g->sm_count * 8 / conc + 1;
     CK(cudaEventRecord(w.ev[0], s), "event");
@@ -508,7 +460,7 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     CK(cudaMemcpyAsync(w.h_ctl, w.ctl.p, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "status copy");
     w.last_grid = grid;
     w.last_block = bt;
-    w.last_worker = warp_worker ? SSSP_WORKER_WARP : SSSP_WORKER_CTA;
+    w.last_worker = SSSP_WORKER_CTA;
     w.last_k0 = k;
     return SSSP_OK;
 }
@@ -628,6 +580,17 @@ void accumulate(sssp_graph* g, Workspace& w, const Ctl& c, int bits) {
     st.total_ms += b;
 }
 
+// An aborted attempt leaves items in the bucket ring and chunks in the hub-split
+// queue (init_run_kernel resets only the counters): wipe both before the
+// workspace is used again (shared by the synchronous retry path and the
+// SSSP_FLAG_ASYNC error path of sssp_get_stats).
+sssp_status clear_after_abort(Workspace& w, cudaStream_t s) {
+    CK(cudaMemsetAsync(w.ring.p, 0xFF, w.ring.bytes, s), "clearing the bucket ring");
+    if (w.tasks.p) CK(cudaMemsetAsync(w.tasks.p, 0, w.tasks.bytes, s), "clearing the split-chunk queue");
+    CK(cudaStreamSynchronize(s), "clearing the bucket ring");
+    return SSSP_OK;
+}
+
 // Inspect a finished attempt.  Returns SSSP_OK and sets *done on success; on a
 // recoverable device status prepares the retry (clears/grows the ring, switches
 // to 64-bit) and leaves *done false; otherwise returns the error.
@@ -639,10 +602,8 @@ sssp_status settle_attempt(sssp_graph* g, Workspace& w, cudaStream_t s, int& bit
         *done = true;
         return SSSP_OK;
     }
-    // aborted attempt: the ring holds leftovers -> clear it before anything else
-    CK(cudaMemsetAsync(w.ring.p, 0xFF, w.ring.bytes, s), "clearing the bucket ring");
-    if (w.tasks.p) CK(cudaMemsetAsync(w.tasks.p, 0, w.tasks.bytes, s), "clearing the split-chunk queue");
-    CK(cudaStreamSynchronize(s), "clearing the bucket ring");
+    sssp_status cst = clear_after_abort(w, s);
+    if (cst) return cst;
     if (status & kStTimeout) return fail(SSSP_ERR_TIMEOUT, "device watchdog expired");
     if (status & kStBug) return fail(SSSP_ERR_CUDA, "internal invariant violated");
     if (status & kStDistOverflow) {
@@ -741,6 +702,12 @@ sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, c
     return st;
 }
 
+void restore_persist(sssp_graph* g) {
+    if (!g->persist_saved) return;
+    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, g->persist_prev);
+    g->persist_saved = false;
+}
+
 sssp_status run_many(sssp_graph* g, const uint32_t* sources, uint32_t k, void* dist_out, bool f32_out,
                      sssp_stream_t stream) {
     if (!g || !dist_out || (k && !sources)) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL argument");
@@ -804,6 +771,7 @@ sssp_status run_many(sssp_graph* g, const uint32_t* sources, uint32_t k, void* d
         cudaEventElapsedTime(&ms, g->bev[0], g->bev[1]);
         g->stats.batch_ms = ms;
     }
+    if (!async) restore_persist(g);
     g->stats.status = st;
     g->busy = false;
     return st;
@@ -821,7 +789,7 @@ void sssp_options_default(sssp_options* o) {
     o->device = 0;
     o->num_buckets = 32;
     o->delta_mode = SSSP_DELTA_DYNAMIC;
-    o->delta_init = 0;             // heuristic C*W/D
+    o->delta_init = 0;             // 0 = heuristic (delta_heuristic; default ring span w_max/B, reading R3)
     o->clip_pct = 65;
     o->settle_head_switches = 8;   // P:215 (reading R7): controller steps between Delta changes
     o->util_lo_pct = 100;          // P:211 (reading R6)
@@ -852,25 +820,30 @@ namespace {
 // of the graph, not of its numbering: the source is mapped in, finalize gathers the
 // output back in caller order, so results are bit-identical.  Auto: on when the
 // in-degree is skewed (max > 64 x average); SSSP_FLAG_RELABEL / SSSP_FLAG_NO_RELABEL
-// force it; SSSP_RELABEL=0/1 in the environment overrides both (A/B).
+// force it.
 sssp_status relabel_graph(sssp_graph* g, const sssp_options& o) {
     const unsigned n = g->n;
     const unsigned long long m = g->m;
     const unsigned aux_grid = (unsigned)g->sm_count * 8;
+    // CUB's item counts are int: graphs beyond INT_MAX vertices keep their numbering
+    if (n > 0x7FFFFFFFu) return SSSP_OK;
     unsigned* indeg = nullptr;
     CK(cudaMalloc(&indeg, (size_t)n * 4), "relabel: in-degrees");
-    cudaMemset(indeg, 0, (size_t)n * 4);
-    indegree_kernel<<<aux_grid, 256>>>(g->d_adj, m, indeg);
     unsigned mx = 0;
     {
         unsigned* d_mx = nullptr;
         void* tmp = nullptr;
         size_t tb = 0;
-        cub::DeviceReduce::Max(tmp, tb, indeg, d_mx, n);
-        cudaMalloc(&d_mx, 4);
-        cudaMalloc(&tmp, tb);
-        cub::DeviceReduce::Max(tmp, tb, indeg, d_mx, n);
-        cudaError_t e = cudaMemcpy(&mx, d_mx, 4, cudaMemcpyDeviceToHost);
+        cudaError_t e = cudaMemset(indeg, 0, (size_t)n * 4);
+        if (e == cudaSuccess) {
+            indegree_kernel<<<aux_grid, 256>>>(g->d_adj, m, indeg);
+            e = cudaGetLastError();
+        }
+        if (e == cudaSuccess) e = cub::DeviceReduce::Max(tmp, tb, indeg, d_mx, (int)n);
+        if (e == cudaSuccess) e = cudaMalloc(&d_mx, 4);
+        if (e == cudaSuccess) e = cudaMalloc(&tmp, tb);
+        if (e == cudaSuccess) e = cub::DeviceReduce::Max(tmp, tb, indeg, d_mx, (int)n);
+        if (e == cudaSuccess) e = cudaMemcpy(&mx, d_mx, 4, cudaMemcpyDeviceToHost);
         cudaFree(tmp);
         cudaFree(d_mx);
         if (e != cudaSuccess) {
@@ -882,7 +855,6 @@ sssp_status relabel_graph(sssp_graph* g, const sssp_options& o) {
     bool on = (double)mx > 64.0 * (double)m / (double)n;
     if (o.flags & SSSP_FLAG_RELABEL) on = true;
     if (o.flags & SSSP_FLAG_NO_RELABEL) on = false;
-    if (const char* e = std::getenv("SSSP_RELABEL")) on = std::atoi(e) != 0;
     if (!on) {
         cudaFree(indeg);
         return SSSP_OK;
@@ -905,17 +877,21 @@ sssp_status relabel_graph(sssp_graph* g, const sssp_options& o) {
     if (e == cudaSuccess) e = cudaMalloc(&deg_new, (size_t)(n + 1) * 8);
     if (e == cudaSuccess) e = cudaMalloc(&off_new, (size_t)(n + 1) * 8);
     if (e == cudaSuccess) e = cudaMalloc(&adj_new, (size_t)m * sizeof(uint2));
-    if (e == cudaSuccess) {
-        cub::DeviceRadixSort::SortPairs(nullptr, tb_sort, key, key_out, iota, old_of_new, (int)n);
-        cub::DeviceScan::ExclusiveSum(nullptr, tb_scan, deg_new, off_new, (int)n + 1);
-        e = cudaMalloc(&tmp, std::max(tb_sort, tb_scan));
-    }
+    if (e == cudaSuccess) e = cub::DeviceRadixSort::SortPairs(nullptr, tb_sort, key, key_out, iota, old_of_new, (int)n);
+    if (e == cudaSuccess) e = cub::DeviceScan::ExclusiveSum(nullptr, tb_scan, deg_new, off_new, (int)n + 1);
+    if (e == cudaSuccess) e = cudaMalloc(&tmp, std::max(tb_sort, tb_scan));
     if (e == cudaSuccess) {
         relabel_keys_kernel<<<aux_grid, 256>>>(indeg, n, key, iota);
-        cub::DeviceRadixSort::SortPairs(tmp, tb_sort, key, key_out, iota, old_of_new, (int)n);
-        cudaMemset(deg_new + n, 0, 8);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess) e = cub::DeviceRadixSort::SortPairs(tmp, tb_sort, key, key_out, iota, old_of_new, (int)n);
+    if (e == cudaSuccess) e = cudaMemset(deg_new + n, 0, 8);
+    if (e == cudaSuccess) {
         relabel_inverse_kernel<<<aux_grid, 256>>>(old_of_new, n, g->d_off, new_of_old, deg_new);
-        cub::DeviceScan::ExclusiveSum(tmp, tb_scan, deg_new, off_new, (int)n + 1);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess) e = cub::DeviceScan::ExclusiveSum(tmp, tb_scan, deg_new, off_new, (int)n + 1);
+    if (e == cudaSuccess) {
         relabel_arcs_kernel<<<aux_grid, 256>>>(old_of_new, new_of_old, n, g->d_off, off_new, g->d_adj, adj_new);
         e = cudaDeviceSynchronize();
     }
@@ -1077,6 +1053,7 @@ sssp_status sssp_graph_destroy(sssp_graph* g) {
     g->ws.clear();
     g->scratch.release();
     g->hostout.release();
+    g->cert.release();
     for (auto& e : g->bev)
         if (e) cudaEventDestroy(e);
     delete g;
@@ -1133,9 +1110,24 @@ sssp_status sssp_get_stats(sssp_graph* g, sssp_stats* out) {
         e = cudaDeviceSynchronize();
         if (e != cudaSuccess) return cuda_fail(e, "async run");
         const unsigned status = w.h_ctl->status;
+        restore_persist(g);
         if (status) {
-            cudaMemset(w.ring.p, 0xFF, w.ring.bytes);
-            cudaDeviceSynchronize();
+            // same cleanup and retry decisions as the synchronous path (settle_attempt):
+            // the next run starts from a clean ring / chunk queue, 64-bit after an overflow
+            sssp_status cst = clear_after_abort(w, (cudaStream_t)0);
+            if (cst) return cst;
+            if ((status & kStDistOverflow) && !g->opts.dist_bits) g->cur_bits = 64;
+            if ((status & kStRingOverflow) && !(status & (kStTimeout | kStBug))) {
+                // grow like the synchronous retry would, so the caller's re-run fits
+                sssp_status gst = ensure_tasks(g, w, w.tcap * 2);
+                if (gst == SSSP_OK) {
+                    const unsigned long long ncap = w.cap * 2;
+                    const int ib = w.ring_item_bytes;
+                    w.ring.release();
+                    gst = ensure_ring(g, w, ib, ncap);
+                }
+                if (gst) return gst;
+            }
             g->stats.status = (status & kStRingOverflow)   ? SSSP_ERR_WORKLIST_OVERFLOW
                               : (status & kStTimeout)      ? SSSP_ERR_TIMEOUT
                               : (status & kStDistOverflow) ? SSSP_ERR_INVALID_ARGUMENT
@@ -1171,6 +1163,83 @@ sssp_status sssp_get_profile(sssp_graph* g, uint64_t* out, uint32_t cap, uint32_
     const Ctl* hc = g->ws.empty() ? nullptr : g->ws[0]->h_ctl;
     for (uint32_t i = 0; i < c; ++i) out[i] = hc ? hc->prof[i] : 0;
     *count = c;
+    return SSSP_OK;
+}
+
+sssp_status sssp_certify(sssp_graph* g, uint32_t source, const void* dist, sssp_certificate* out,
+                         sssp_stream_t stream) {
+    if (!g || !dist || !out) return fail(SSSP_ERR_INVALID_ARGUMENT, "NULL argument");
+    if (source >= g->n) return fail(SSSP_ERR_INVALID_ARGUMENT, "source >= n");
+    if (g->busy || g->async_pending) return fail(SSSP_ERR_BUSY, "a run is in flight on this handle");
+    DeviceGuard dg(g->device);
+    std::memset(out, 0, sizeof(*out));
+    cudaStream_t s = (cudaStream_t)stream;
+    const size_t esz = g->f32 ? 4 : 8;
+    bool is_dev = false;
+    sssp_status st = classify_out(g, dist, &is_dev);
+    if (st) return st;
+    if (!is_dev) {  // host vector: stage it on the device
+        if (!g->hostout.p) {
+            CK(cudaMalloc(&g->hostout.p, (size_t)g->n * 8), "allocating the staging buffer");
+            g->hostout.bytes = (size_t)g->n * 8;
+        }
+        CK(cudaMemcpyAsync(g->hostout.p, dist, (size_t)g->n * esz, cudaMemcpyHostToDevice, s), "staging dist");
+        dist = g->hostout.p;
+    }
+    if (!g->cert.p) {
+        CK(cudaMalloc(&g->cert.p, sizeof(CertState)), "allocating the certificate state");
+        g->cert.bytes = sizeof(CertState);
+    }
+    CertState h{};
+    h.first_violated = h.first_unanchored = ~0ull;
+    CK(cudaMemcpyAsync(g->cert.p, &h, sizeof(h), cudaMemcpyHostToDevice, s), "certificate state");
+    Workspace& w = *g->ws[0];
+    unsigned long long* dint = (unsigned long long*)w.dist.p;  // 8n bytes of scratch (no run in flight)
+    unsigned* anchors = (unsigned*)w.expanded.p;              // n bits
+    CertState* dst = (CertState*)g->cert.p;
+    const unsigned src_int = g->h_perm.empty() ? source : g->h_perm[source];
+    const unsigned grid = (unsigned)g->sm_count * 8;
+    auto run_rounds = [&](auto kf) -> sssp_status {
+        constexpr bool kF = decltype(kf)::value;
+        certify_scatter_kernel<kF><<<grid, 256, 0, s>>>(dist, dint, g->d_perm, g->n, source, anchors, dst);
+        certify_arcs_kernel<kF><<<grid, 256, 0, s>>>(dint, g->d_off, g->d_adj, g->n, src_int, anchors, dst);
+        CK(cudaGetLastError(), "certificate kernels");
+        CK(cudaMemcpyAsync(&h, dst, sizeof(h), cudaMemcpyDeviceToHost, s), "certificate state");
+        CK(cudaStreamSynchronize(s), "certificate");
+        // tight arcs between equal distances: anchor to a fixed point (at most n rounds)
+        if (h.equal_tight) {
+            for (uint32_t r = 0; r < g->n; ++r) {
+                CK(cudaMemsetAsync(&dst->changed, 0, 8, s), "certificate flag");
+                certify_equal_kernel<kF><<<grid, 256, 0, s>>>(dint, g->d_off, g->d_adj, g->n, anchors, dst);
+                CK(cudaMemcpyAsync(&h, dst, sizeof(h), cudaMemcpyDeviceToHost, s), "certificate state");
+                CK(cudaStreamSynchronize(s), "certificate");
+                out->fixpoint_rounds = r + 1;
+                if (!h.changed) break;
+            }
+        }
+        certify_check_kernel<kF><<<grid, 256, 0, s>>>(dint, g->d_off, g->n, anchors, dst);
+        CK(cudaGetLastError(), "certificate kernels");
+        CK(cudaMemcpyAsync(&h, dst, sizeof(h), cudaMemcpyDeviceToHost, s), "certificate state");
+        CK(cudaStreamSynchronize(s), "certificate");
+        return SSSP_OK;
+    };
+    st = g->f32 ? run_rounds(std::true_type{}) : run_rounds(std::false_type{});
+    if (st) return st;
+    auto to_caller = [&](unsigned long long iv) -> uint64_t {
+        if (iv == ~0ull || g->h_perm.empty()) return iv;
+        for (uint32_t v = 0; v < g->n; ++v)
+            if (g->h_perm[v] == iv) return v;
+        return iv;
+    };
+    out->source_ok = h.source_bad == 0 ? 1u : 0u;
+    out->violated_arcs = h.violated;
+    out->first_violated_tail = to_caller(h.first_violated);
+    out->unanchored = h.unanchored;
+    out->first_unanchored = to_caller(h.first_unanchored);
+    out->bad_markers = h.bad_inf;
+    out->reachable = h.reach_v;
+    out->reach_edges = h.reach_e;
+    out->exact = (out->source_ok && !h.violated && !h.unanchored && !h.bad_inf) ? 1u : 0u;
     return SSSP_OK;
 }
 

@@ -34,11 +34,24 @@ def test_library_exports_every_declared_symbol():
     assert set(declared_functions()) == bound
 
 
-def test_nm_shows_only_c_symbols():
+@pytest.mark.parametrize("variant", ["", "fuzz"])
+def test_nm_shows_only_c_symbols(variant):
     import subprocess
-    out = subprocess.run(["nm", "-D", "--defined-only", sssp.LIB_PATH], capture_output=True, text=True).stdout
+    from paper_conf_ppopp_wangfl21_b200 import _build
+    out = subprocess.run(["nm", "-D", "--defined-only", _build.variant_path(variant)], capture_output=True,
+                         text=True).stdout
     exported = {l.split()[-1] for l in out.splitlines() if " T " in l and l.split()[-1].startswith("sssp_")}
     assert exported == set(declared_functions())
+
+
+def test_fuzz_variant_loads_and_differs():
+    """libsssp_fuzz.so (-DSSSP_FUZZ) is a separate build of the same ABI: it carries the
+    delay-injection points (more SASS), the product library does not."""
+    from paper_conf_ppopp_wangfl21_b200 import _build
+    L = sssp.lib("fuzz")
+    for name in declared_functions():
+        assert hasattr(L, name), name
+    assert os.path.getsize(_build.variant_path("fuzz")) != os.path.getsize(_build.LIB)
 
 
 def _c_struct_sizes():
@@ -50,8 +63,9 @@ def _c_struct_sizes():
 #include <stddef.h>
 #include "sssp.h"
 int main(void){
-  printf("%zu %zu %zu %zu %zu %zu\n", sizeof(sssp_options), sizeof(sssp_stats), sizeof(sssp_trace_entry),
-         offsetof(sssp_options, ring_items), offsetof(sssp_stats, kernel_ms), offsetof(sssp_options, active_init));
+  printf("%zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(sssp_options), sizeof(sssp_stats), sizeof(sssp_trace_entry),
+         offsetof(sssp_options, ring_items), offsetof(sssp_stats, kernel_ms), offsetof(sssp_options, active_init),
+         sizeof(sssp_certificate), offsetof(sssp_certificate, fixpoint_rounds));
   return 0; }
 '''
     with tempfile.TemporaryDirectory() as d:
@@ -63,7 +77,9 @@ int main(void){
 
 
 def test_struct_layouts_match_python_mirror():
-    so, ss, st, off_ring, off_kms, off_act = _c_struct_sizes()
+    so, ss, st, off_ring, off_kms, off_act, sc, off_fix = _c_struct_sizes()
+    assert sc == ctypes.sizeof(sssp.sssp_certificate)
+    assert off_fix == sssp.sssp_certificate.fixpoint_rounds.offset
     assert so == ctypes.sizeof(sssp.sssp_options)
     assert ss == ctypes.sizeof(sssp.sssp_stats)
     assert st == ctypes.sizeof(sssp.sssp_trace_entry)
@@ -78,7 +94,8 @@ def test_option_defaults_follow_the_paper():
     assert o.num_buckets == 32          # P:174 "a fixed number of 32 buckets"
     assert o.clip_pct == 65             # P:207 "at least 65%"
     assert o.delta_mode == sssp.SSSP_DELTA_DYNAMIC
-    assert o.delta_init == 0            # heuristic C*W/D
+    assert o.delta_init == 0            # 0 = heuristic: ring span w_max/B by default (reading R3)
+    assert o.delta_heuristic == sssp.SSSP_DELTA_H_RING_SPAN
     assert o.settle_head_switches >= 1  # P:215 "a fixed number of head bucket switches"
 
 
@@ -133,6 +150,32 @@ def test_create_without_gpu_fails_loudly():
     with pytest.raises(sssp.SSSPError) as e:
         sssp.Graph(np.array([0, 1], dtype=np.uint64), np.array([0], dtype=np.uint32), np.array([1], dtype=np.uint32))
     assert e.value.status == 9  # SSSP_ERR_NO_DEVICE: no CPU fallback
+
+
+def test_python_binding_refuses_mistyped_inputs():
+    """tensors / arrays of the wrong dtype are converted with range checks or
+    refused, never reinterpreted (an int64 col read as uint32 pairs, float64 weights)."""
+    import numpy as np
+    import torch
+    p, keep = sssp._as_host_or_dev(torch.tensor([1, 2, 3], dtype=torch.int64), np.uint32, "col")
+    assert keep.dtype == torch.int32 and keep.tolist() == [1, 2, 3]
+    p, keep = sssp._as_host_or_dev(torch.tensor([0, 5], dtype=torch.int64), np.uint64, "row_offsets")
+    assert keep.dtype == torch.int64
+    with pytest.raises(ValueError):
+        sssp._as_host_or_dev(torch.tensor([1 << 33], dtype=torch.int64), np.uint32, "col")
+    with pytest.raises(ValueError):
+        sssp._as_host_or_dev(torch.tensor([-1], dtype=torch.int32), np.uint32, "col")
+    with pytest.raises(TypeError):
+        sssp._as_host_or_dev(torch.tensor([1.0], dtype=torch.float64), np.uint32, "w")
+    with pytest.raises(TypeError):
+        sssp._as_host_or_dev(torch.tensor([1.0], dtype=torch.float64), np.float32, "w")
+    with pytest.raises(TypeError):
+        sssp._as_host_or_dev(np.array([1.5]), np.float32, "w")
+    with pytest.raises(ValueError):
+        sssp._as_host_or_dev(np.array([1 << 40], dtype=np.int64), np.uint32, "w")
+    p, keep = sssp._as_host_or_dev(np.array([1, 2], dtype=np.int64), np.uint32, "w")
+    assert keep.dtype == np.uint32
+    assert sssp._is_float(np.array([1.5])) and not sssp._is_float(np.array([1]))
 
 
 def test_package_does_not_import_oracle():

@@ -25,17 +25,17 @@ import paper_conf_ppopp_wangfl21_b200 as sssp  # noqa: E402
 INF = np.uint64(0xFFFFFFFFFFFFFFFF)
 
 
-def gpu_dist(g, s, **opt):
-    G = sssp.Graph.from_csr(g, **opt)
+def gpu_dist(g, s, variant="", **opt):
+    G = sssp.Graph.from_csr(g, variant=variant, **opt)
     d = sssp.to_u64(G.run(int(s)))
     st = G.stats()
     G.close()
     return d, st
 
 
-def check(g, s, **opt):
+def check(g, s, variant="", **opt):
     ref, V, E = oracle.dijkstra(g, int(s))
-    d, st = gpu_dist(g, s, **opt)
+    d, st = gpu_dist(g, s, variant=variant, **opt)
     bad = np.flatnonzero(d != ref)
     assert bad.size == 0, f"{bad.size} mismatches, first v={bad[:5]} gpu={d[bad[:5]]} ref={ref[bad[:5]]} opt={opt}"
     assert st["reachable"] == V and st["reach_edges"] == E
@@ -54,13 +54,13 @@ def test_golden_fixtures_on_gpu(name):
 
 
 @pytest.mark.parametrize("name", golden_names())
-def test_golden_fixtures_warp_worker(name):
+def test_golden_fixtures_fuzzed(name):
+    """The schedule-fuzzing build (hash-driven delays at reserve/publish/claim/complete/head-CAS)."""
     fx = load_golden(name)
     g = gg.from_arcs(fx["n"], fx["arcs"])
-    d, st = gpu_dist(g, fx["source"], worker=sssp.SSSP_WORKER_WARP)
+    d, st = gpu_dist(g, fx["source"], variant="fuzz")
     assert [int(x) for x in d] == fx["dist"]
     assert st["reachable"] == fx["V"] and st["reach_edges"] == fx["E"]
-    assert st["worker"] == sssp.SSSP_WORKER_WARP
 
 
 @pytest.mark.parametrize("name", golden_names())
@@ -84,11 +84,13 @@ def test_relabel_auto_on_skewed_graphs_only():
 
 
 def test_worker_selection():
-    # AUTO = the CTA worker (measured faster everywhere, D12); WARP on request
+    # AUTO = the CTA worker; the warp-granular ablation was removed (D12)
     rmat = gg.make("rmat", scale_down=10)
     s = gg.config_sources("rmat", rmat, 1)[0]
     assert check(rmat, s)["worker"] == sssp.SSSP_WORKER_CTA
-    assert check(rmat, s, worker=sssp.SSSP_WORKER_WARP)["worker"] == sssp.SSSP_WORKER_WARP
+    with pytest.raises(sssp.SSSPError) as e:
+        sssp.Graph.from_csr(rmat, worker=2)
+    assert e.value.status == 1
 
 
 def test_u32_overflow_reruns_in_64_bits():
@@ -117,7 +119,7 @@ def test_random_small_graphs():
         arcs = list(zip(rng.integers(0, n, m), rng.integers(0, n, m), rng.integers(0, wmax, m, endpoint=True)))
         g = gg.from_arcs(n, arcs)
         check(g, int(rng.integers(0, n)))
-        check(g, int(rng.integers(0, n)), worker=sssp.SSSP_WORKER_WARP)
+        check(g, int(rng.integers(0, n)), variant="fuzz")
 
 
 def test_config_grid64():
@@ -155,16 +157,7 @@ PERTURB = [
     dict(flags=sssp.SSSP_FLAG_NO_WARP_LOCAL), dict(flags=sssp.SSSP_FLAG_WARP_LOCAL, local_max=1, grid_ctas=2), dict(block_threads=1024),
     # relaxation filter on the 16-bit upper-bound array instead of dist itself
     dict(flags=sssp.SSSP_FLAG_FILTER16), dict(flags=sssp.SSSP_FLAG_FILTER16, dist_bits=64),
-    # worker granularity (D12): each worker forced on every graph, and the warp
-    # worker under the schedule extremes (one CTA, 64-bit, tiny rings, 1-arc / no hub
-    # chunks, 2 buckets, Delta = 1, tracing, static huge Delta)
-    dict(worker=sssp.SSSP_WORKER_WARP), dict(worker=sssp.SSSP_WORKER_CTA),
-    dict(worker=sssp.SSSP_WORKER_WARP, grid_ctas=1), dict(worker=sssp.SSSP_WORKER_WARP, dist_bits=64),
-    dict(worker=sssp.SSSP_WORKER_WARP, ring_items=64), dict(worker=sssp.SSSP_WORKER_WARP, split_degree=1),
-    dict(worker=sssp.SSSP_WORKER_WARP, split_degree=0xFFFFFFFF), dict(worker=sssp.SSSP_WORKER_WARP, num_buckets=2),
-    dict(worker=sssp.SSSP_WORKER_WARP, delta_mode=1, delta_init=1),
-    dict(worker=sssp.SSSP_WORKER_WARP, delta_mode=1, delta_init=1 << 30),
-    dict(worker=sssp.SSSP_WORKER_WARP, flags=sssp.SSSP_FLAG_TRACE),
+    dict(worker=sssp.SSSP_WORKER_CTA),
     # locality relabeling (D15) forced on / off, with the 64-bit and Near-Far paths
     dict(flags=sssp.SSSP_FLAG_RELABEL), dict(flags=sssp.SSSP_FLAG_NO_RELABEL),
     dict(flags=sssp.SSSP_FLAG_RELABEL, dist_bits=64),
@@ -175,11 +168,37 @@ PERTURB = [
 @pytest.mark.parametrize("opt", PERTURB, ids=lambda o: ",".join(f"{k}={v}" for k, v in o.items()))
 @pytest.mark.parametrize("config", ["road", "rmat", "er"])
 def test_schedule_perturbation(config, opt):
-    g = gg.make(config, scale_down=10 if config != "road" else 10)
+    g = gg.make(config, scale_down=10)
     s = gg.config_sources(config, g, 1)[0]
-    st = check(g, s, **opt)
-    if opt.get("ring_items"):
-        assert st["retries"] >= 0
+    check(g, s, **opt)
+
+
+# the same matrix on the schedule-fuzzing build (libsssp_fuzz.so, -DSSSP_FUZZ): hash-driven
+# 32 ns - 4 us delays at the reserve / publish / claim / pop / complete / head-CAS / chunk points
+# reorder the worklist protocol's steps far more than the natural schedule does
+FUZZ = [dict(), dict(grid_ctas=3), dict(block_threads=128), dict(block_threads=512), dict(num_buckets=2),
+        dict(dist_bits=64), dict(active_init=32), dict(batch_min=1), dict(ring_items=64),
+        dict(flags=sssp.SSSP_FLAG_NO_LOCAL), dict(local_max=1), dict(split_degree=1), dict(split_degree=3, grid_ctas=3),
+        dict(delta_mode=1, delta_init=1), dict(delta_mode=1, delta_init=1 << 30), dict(flags=sssp.SSSP_FLAG_ADAPT_ACTIVE),
+        dict(settle_head_switches=1, util_lo_pct=1000, util_hi_pct=2000), dict(flags=sssp.SSSP_FLAG_TRACE),
+        dict(flags=sssp.SSSP_FLAG_WARP_LOCAL, local_max=1, grid_ctas=2), dict(concurrent_sources=1)]
+
+
+@pytest.mark.parametrize("opt", FUZZ, ids=lambda o: ",".join(f"{k}={v}" for k, v in o.items()) or "default")
+@pytest.mark.parametrize("config", ["road", "rmat", "er"])
+def test_fuzzed_schedule(config, opt):
+    g = gg.make(config, scale_down=10)
+    for s in gg.config_sources(config, g, 2):
+        check(g, s, variant="fuzz", **opt)
+
+
+def test_fuzzed_concurrent_batch():
+    g = gg.make("road", scale_down=9)
+    srcs = gg.config_sources("road", g, 6)
+    G = sssp.Graph.from_csr(g, variant="fuzz", concurrent_sources=3, ring_items=256)
+    D = G.run_batch(srcs)
+    for i, s in enumerate(srcs):
+        assert np.array_equal(sssp.to_u64(D[i]), oracle.dijkstra(g, int(s))[0])
 
 
 def test_tiny_ring_without_retry_reports_overflow():
@@ -293,33 +312,60 @@ def test_full_size_config(config):
     g = gg.make(config)
     s = int(gg.config_sources(config, g, 1)[0])
     ref, V, E = oracle.dijkstra(g, s)
-    # the bench's launch configuration (auto worker) and each worker forced
-    runs = [dict(worker=w) for w in (sssp.SSSP_WORKER_AUTO, sssp.SSSP_WORKER_CTA, sssp.SSSP_WORKER_WARP)]
-    runs += [dict(flags=sssp.SSSP_FLAG_NO_RELABEL if config == "rmat" else sssp.SSSP_FLAG_RELABEL)]
-    for opt in runs:
-        d, st = gpu_dist(g, s, **opt)
+    # the bench's launch configuration, 64-bit distances, and the other relabeling choice
+    # (relabeling happens at create time: its own handle)
+    G = sssp.Graph.from_csr(g)
+    H = sssp.Graph.from_csr(g, flags=sssp.SSSP_FLAG_NO_RELABEL if config == "rmat" else sssp.SSSP_FLAG_RELABEL)
+    assert G.info()["relabeled"] != H.info()["relabeled"]
+    for X, opt in ((G, dict()), (G, dict(dist_bits=64)), (H, dict())):
+        if opt:
+            X.set_options(**opt)
+        out = X.run(s)
+        st = X.stats()
+        d = sssp.to_u64(out)
         bad = np.flatnonzero(d != ref)
         assert bad.size == 0, f"{opt}: {bad.size} mismatches, first v={bad[:5]}"
         assert st["reachable"] == V and st["reach_edges"] == E
-        assert st["dist_bits"] == 32
+        assert st["dist_bits"] == opt.get("dist_bits", 32)
+        c = X.certify(s, out)
+        assert c["exact"] == 1 and c["reachable"] == V and c["reach_edges"] == E
 
 
-def test_full_size_batch_sampled():
-    """Config 5 at full size in bench.py's launch configuration (RMAT-24, 2 sources in
-    flight): a seeded sample of the 512 batch sources, each row compared with the oracle,
-    plus the rank-partition the multi-GPU bench uses (sources[r::G])."""
+@pytest.mark.timeout(1800)
+def test_full_size_batch_every_source():
+    """Config 5 at full size in bench.py's launch configuration (RMAT-24, all 512 sources,
+    2 in flight, through the same rank loop as the multi-GPU bench): EVERY row passes the GPU
+    certificate (sssp_certify: no violated arc, every finite vertex reachable through tight
+    arcs, dist[s] = 0, reach counts = the run's), and a seeded half of the rows (256) is
+    compared element by element with the oracle, streamed over a pool of host threads."""
+    import concurrent.futures as cf
+    import os
+    from paper_conf_ppopp_wangfl21_b200.distributed import run_batch_distributed
     g = gg.make("batch")
     srcs = gg.sources(g, 512, gg.CONFIGS["batch"]["source_seed"])
-    rng = np.random.default_rng(5)
-    pick = np.sort(rng.choice(512, size=6, replace=False))
-    sample = srcs[pick]
+    assert len(set(srcs.tolist())) == 512
     G = sssp.Graph.from_csr(g, concurrent_sources=2)
-    D = G.run_batch(sample)
-    assert G.stats()["concurrency"] == 2
-    for i, s in enumerate(sample):
-        assert np.array_equal(sssp.to_u64(D[i]), oracle.dijkstra(g, int(s))[0]), f"source {int(s)}"
+    D = torch.empty((512, g.n), dtype=torch.int64, device="cuda")
+    res = run_batch_distributed(G, srcs, out=D)
+    assert res["stats"]["runs"] == 512 and G.stats()["concurrency"] == 2
+    E_cert = 0
+    for i, s in enumerate(srcs):
+        c = G.certify(int(s), D[i])
+        assert c["exact"] == 1, f"source {int(s)}: {c}"
+        E_cert += c["reach_edges"]
+    assert res["stats"]["reach_edges"] == E_cert      # the run's own E_dij agrees with the certified rows
+    rng = np.random.default_rng(5)
+    half = np.sort(rng.choice(512, size=256, replace=False))
+    workers = max(1, min(16, (os.cpu_count() or 2) - 1))
+    with cf.ThreadPoolExecutor(workers) as ex:
+        futs = {ex.submit(oracle.dijkstra, g, int(srcs[i])): i for i in half}
+        for f in cf.as_completed(futs):
+            i = futs[f]
+            ref, V, E = f.result()
+            row = sssp.to_u64(D[i])
+            assert np.array_equal(row, ref), f"source {int(srcs[i])}"
     parts = [srcs[r::8] for r in range(8)]
-    assert sorted(np.concatenate(parts).tolist()) == sorted(srcs.tolist()) and len(set(srcs.tolist())) == 512
+    assert sorted(np.concatenate(parts).tolist()) == sorted(srcs.tolist())
 
 
 def test_run_batch_distributed_single_rank():
@@ -327,7 +373,8 @@ def test_run_batch_distributed_single_rank():
     g = gg.make("rmat", scale_down=10)
     srcs = gg.sources(g, 5, seed=5)
     G = sssp.Graph.from_csr(g)
-    out = run_batch_distributed(G, srcs, gather=True)
+    out = run_batch_distributed(G, srcs, gather_to=0)
+    assert out["max_ms"] > 0 and out["max_ms"] == out["local_ms"]
     full = sssp.to_u64(out["full"])
     for i, s in enumerate(srcs):
         assert np.array_equal(full[i], oracle.dijkstra(g, int(s))[0])
@@ -508,3 +555,122 @@ def test_bench_json_contract_small_config():
     assert line["roofline"]["peak"] > 0 and 0 < line["roofline"]["frac"] < 1
     assert line["cpu_baseline"]["kind"] == "oracle" and line["cpu_baseline"]["cores"] == 1
     assert "sm_mhz" in line["clocks"]
+
+
+# ----------------------------------------------------------------- GPU certificate (sssp_certify)
+def _perturbations(g, s, ref, rng):
+    """Corruptions of the exact vector that a complete certificate must reject."""
+    fin = np.flatnonzero((ref != INF) & (np.arange(g.n) != s))
+    unr = np.flatnonzero(ref == INF)
+    out = []
+    d = ref.copy(); d[s] = 1; out.append(d)                              # (i)
+    for v in rng.choice(fin, size=min(3, fin.size), replace=False) if fin.size else []:
+        if ref[v] > 0:
+            d = ref.copy(); d[v] -= 1; out.append(d)                     # too small: no tight path
+        d = ref.copy(); d[v] += 1; out.append(d)                         # too large: an arc violated
+        d = ref.copy(); d[v] = INF; out.append(d)                        # finite -> unreachable
+    for v in rng.choice(unr, size=min(2, unr.size), replace=False) if unr.size else []:
+        d = ref.copy(); d[v] = 7; out.append(d)                          # unreachable -> finite
+    return out
+
+
+def test_certificate_accepts_exact_and_rejects_perturbed():
+    rng = np.random.default_rng(11)
+    graphs = []
+    for t in range(12):
+        n = int(rng.integers(2, 200))
+        m = int(rng.integers(0, 6 * n))
+        wmax = int(rng.choice([0, 1, 3, 1000, 0xFFFFFFFF]))
+        arcs = list(zip(rng.integers(0, n, m), rng.integers(0, n, m), rng.integers(0, wmax, m, endpoint=True)))
+        graphs.append((gg.from_arcs(n, arcs), {}))
+    r = gg.make("rmat", scale_down=12)
+    graphs += [(r, {}), (r, dict(flags=sssp.SSSP_FLAG_RELABEL)), (gg.make("road", scale_down=12), {})]
+    for g, opt in graphs:
+        G = sssp.Graph.from_csr(g, **opt)
+        s = int(rng.integers(0, g.n))
+        ref, V, E = oracle.dijkstra(g, s)
+        c = G.certify(s, ref)
+        assert c["exact"] == 1 and c["reachable"] == V and c["reach_edges"] == E, c
+        dev = G.run(s)
+        assert G.certify(s, dev)["exact"] == 1
+        for d in _perturbations(g, s, ref, rng):
+            c = G.certify(s, d)
+            assert c["exact"] == 0, (c, opt)
+            assert oracle.certify(g, s, d) != 0          # the CPU certificate agrees
+
+
+def test_certificate_zero_weight_fixpoint():
+    # a zero-weight chain hanging off the source and a zero-weight cycle that is NOT reachable
+    # but claims the same distance as a reachable vertex: only the fixpoint tells them apart
+    n = 8
+    arcs = [(0, 1, 5), (1, 2, 0), (2, 3, 0), (3, 4, 0), (5, 6, 0), (6, 5, 0), (0, 7, 3)]
+    g = gg.from_arcs(n, arcs)
+    G = sssp.Graph.from_csr(g)
+    ref, _, _ = oracle.dijkstra(g, 0)
+    c = G.certify(0, ref)
+    assert c["exact"] == 1 and c["fixpoint_rounds"] >= 3
+    d = ref.copy(); d[5] = d[6] = 5                                     # self-supporting zero cycle
+    c = G.certify(0, d)
+    assert c["exact"] == 0 and c["unanchored"] == 2 and c["first_unanchored"] == 5
+    assert oracle.certify(g, 0, d) != 0
+
+
+def test_certificate_float_graph():
+    g = gg.make("rmat", scale_down=12)
+    wf = gg.float_weights(g, 0.0, 1.0, seed=3)
+    s = int(gg.config_sources("rmat", g, 1)[0])
+    G = sssp.Graph.from_csr(g, weights=wf)
+    d = G.run(s)
+    assert G.certify(s, d)["exact"] == 1
+    h = d.cpu().numpy().copy()
+    v = int(np.flatnonzero(np.isfinite(h) & (h > 0))[0])
+    h[v] = np.nextafter(h[v], np.float32(0))
+    assert G.certify(s, h)["exact"] == 0
+
+
+# ----------------------------------------------------------------- ASYNC error path (ADVICE r1)
+def test_async_overflow_then_exact_rerun():
+    g = gg.make("rmat", scale_down=8)
+    s = int(gg.config_sources("rmat", g, 1)[0])
+    G = sssp.Graph.from_csr(g, flags=sssp.SSSP_FLAG_ASYNC, ring_items=64, split_degree=1)
+    G.run(s)
+    torch.cuda.synchronize()
+    with pytest.raises(sssp.SSSPError) as e:
+        G.stats()
+    assert e.value.status == 5
+    # leftovers of the aborted run (ring items, hub chunks) must not leak into the next run
+    G.set_options(flags=0, ring_items=64, split_degree=1)
+    assert np.array_equal(sssp.to_u64(G.run(s)), oracle.dijkstra(g, s)[0])
+    G.set_options(flags=sssp.SSSP_FLAG_ASYNC, ring_items=0, split_degree=1)
+    out = G.run(s)
+    torch.cuda.synchronize()
+    assert G.stats()["status"] == 0
+    assert np.array_equal(sssp.to_u64(out), oracle.dijkstra(g, s)[0])
+
+
+def test_async_dist_overflow_switches_to_64_bits():
+    n = 10
+    g = gg.from_arcs(n, [(i, i + 1, 0xFFFFFFFF) for i in range(n - 1)] + [(0, 5, 7)])
+    G = sssp.Graph.from_csr(g, flags=sssp.SSSP_FLAG_ASYNC)
+    G.run(0)
+    torch.cuda.synchronize()
+    with pytest.raises(sssp.SSSPError):
+        G.stats()
+    out = G.run(0)
+    torch.cuda.synchronize()
+    st = G.stats()
+    assert st["status"] == 0 and st["dist_bits"] == 64
+    assert np.array_equal(sssp.to_u64(out), oracle.dijkstra(g, 0)[0])
+
+
+def test_python_out_checks():
+    g = gg.make("grid64")
+    G = sssp.Graph.from_csr(g)
+    with pytest.raises(TypeError):
+        G.run(0, out=torch.empty(g.n, dtype=torch.int32, device="cuda"))
+    with pytest.raises(ValueError):
+        G.run(0, out=torch.empty(g.n - 1, dtype=torch.int64, device="cuda"))
+    with pytest.raises(ValueError):
+        G.run(0, out=torch.empty((g.n, 2), dtype=torch.int64, device="cuda")[:, 0])
+    with pytest.raises(ValueError):
+        G.run_batch([0, 1], out=torch.empty(g.n, dtype=torch.int64, device="cuda"))
