@@ -526,7 +526,7 @@ __device__ __forceinline__ unsigned take_chunk(const Params<DistT>& p, SplitTask
 // --------------------------------------------------------------- shared memory
 constexpr size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
 
-template <typename DistT, int BT, int EPT, int IPT = 1>
+template <typename DistT, int BT, int EPT>
 struct Smem {
     using Raw = typename ItemT<DistT>::Raw;
     // staged ring pushes of one batch (beyond this, warps publish directly)
@@ -534,13 +534,14 @@ struct Smem {
     static constexpr int kStage = STAGE_MULT * BT * EPT / 2;
     static constexpr size_t o_arc = 0;                                        // (no arc window)
     static constexpr size_t o_items = 0;                                      // Raw[kStage] staged pushes
-    static constexpr size_t o_ebeg = o_items + align16((size_t)kStage * sizeof(Raw));  // u64[BT*IPT] row begin
-    static constexpr size_t o_d = o_ebeg + (size_t)BT * IPT * 8;              // DistT[BT*IPT] item distance
-    static constexpr size_t o_ld = o_d + align16((size_t)BT * IPT * sizeof(DistT)); // DistT[BT] kept children
+    // per expanded item (compacted: items with at least one arc, in scan order)
+    static constexpr size_t o_ebeg = o_items + align16((size_t)kStage * sizeof(Raw));  // u64[BT] row begin - scan
+    static constexpr size_t o_d = o_ebeg + (size_t)BT * 8;                    // DistT[BT] item distance
+    static constexpr size_t o_ld = o_d + align16((size_t)BT * sizeof(DistT));  // DistT[BT] kept children
     static constexpr size_t o_owner = o_ld + align16((size_t)BT * sizeof(DistT));  // (unused)
     static constexpr size_t o_rank = o_owner;                                 // u16[kStage]
-    static constexpr size_t o_scan = o_rank + align16((size_t)kStage * 2);    // u32[BT*IPT]
-    static constexpr size_t o_lv = o_scan + align16((size_t)BT * IPT * 4);    // u32[BT] kept children
+    static constexpr size_t o_scan = o_rank + align16((size_t)kStage * 2);    // u32[BT+1] arc offsets, sentinel E
+    static constexpr size_t o_lv = o_scan + align16((size_t)(BT + 1) * 4);    // u32[BT] kept children
     static constexpr size_t o_soff = o_lv + align16((size_t)BT * 4);          // u8[kStage]
     // warp-local continuation queues: kWQ {vertex, distance, row begin, degree} per warp
     // (the row is fetched when the child is found, so a hop starts with its arc loads)
@@ -567,17 +568,16 @@ template <typename DistT, int BT, int EPT, int MINB, bool PIPE, bool kF, bool WL
 __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<DistT> p) {
     // items per thread: one (batches of two items per thread, to pay the per-batch round
     // trips half as often, measured slower -- ER 13.1 vs 11.4 ms -- from register spills)
-    constexpr int IPT = 1;
     using IT = ItemT<DistT>;
     using Raw = typename IT::Raw;
-    using L = Smem<DistT, BT, EPT, IPT>;
+    using L = Smem<DistT, BT, EPT>;
     constexpr int kStage = L::kStage;
     constexpr int kWarps = BT / 32;
     constexpr unsigned long long kInf = (unsigned long long)DistInf<DistT>::value;
 
     extern __shared__ __align__(16) unsigned char smem[];
     Raw* s_items = (Raw*)(smem + L::o_items);
-    unsigned long long* s_ebeg = (unsigned long long*)(smem + L::o_ebeg);
+    unsigned long long* s_eadj = (unsigned long long*)(smem + L::o_ebeg);  // row begin - arc offset
     DistT* s_d = (DistT*)(smem + L::o_d);
     DistT* s_ld = (DistT*)(smem + L::o_ld);
     unsigned short* s_rank = (unsigned short*)(smem + L::o_rank);
@@ -593,8 +593,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
 
     __shared__ unsigned s_cnt[kMaxBuckets];
     __shared__ unsigned long long s_base[kMaxBuckets];
-    __shared__ unsigned s_wsum[kWarps];
-    __shared__ unsigned s_total, s_E, s_got, s_slot, s_lnext, s_direct, s_task, s_ahead;
+    __shared__ unsigned s_wsum[kWarps], s_wnz[kWarps];
+    __shared__ unsigned s_total, s_E, s_NZ, s_got, s_slot, s_lnext, s_direct, s_task, s_ahead;
     __shared__ int s_cmd;
     __shared__ unsigned long long s_idx;
     __shared__ Head s_head;
@@ -602,6 +602,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const unsigned lt_mask = lanemask_lt();
+    const unsigned le_mask = lt_mask | (1u << lane);
     const unsigned nbm = p.nb - 1;
     const unsigned local_max = p.local_max < (unsigned)BT ? p.local_max : (unsigned)BT;
     unsigned long long c_vert = 0, c_edges = 0, c_push = 0, c_stale = 0, c_local = 0;  // thread 0
@@ -645,7 +646,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 unsigned long long idx = 0;
                 Head hd;
                 bool tk;
-                const unsigned g = claim_batch<DistT, BT * IPT>(p, lane, sl, idx, hd, st, tk);
+                const unsigned g = claim_batch<DistT, BT>(p, lane, sl, idx, hd, st, tk);
                 if (st) {
                     cmd = CMD_EXIT;
                 } else if (g) {
@@ -696,15 +697,11 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         // ------------------------------------------------------------ pop + stale check
         const Head hd = s_head;
         const unsigned hs = meta_hs(hd.meta), k = meta_k(hd.meta);
-        unsigned degs[IPT];
-        bool lives[IPT];
-        unsigned fword[IPT], fbit[IPT];  // expansion-bitmap word before our atomicOr (consumed at batch end)
-#pragma unroll
-        for (int r = 0; r < IPT; ++r) {
-            degs[r] = 0;
-            lives[r] = false;
-            fword[r] = fbit[r] = 0;
-        }
+        unsigned deg = 0;               // arcs this thread's item contributes to the batch
+        bool live = false;              // the item is expanded (not stale)
+        unsigned long long my_b = 0;    // its row begin
+        unsigned long long my_d = 0;    // its distance
+        unsigned fword = 0, fbit = 0;   // expansion-bitmap word before our atomicOr (consumed at batch end)
         if (is_task) {
             // a hub-split chunk: one vertex, len arcs, charged to the slot it carries
             if (tid == 0) {
@@ -718,10 +715,10 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     st_release_u32(&tp->len, 0u);  // free the slot after the read
                     const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
                     if (cur >= d) {  // stale chunks (v improved since) are dropped
-                        degs[0] = len;
-                        s_ebeg[0] = b;
-                        s_d[0] = (DistT)d;
-                        lives[0] = true;
+                        deg = len;
+                        my_b = b;
+                        my_d = d;
+                        live = true;
                     }
                 }
             }
@@ -749,26 +746,18 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     const unsigned long long b = ld_stream_u64(p.off + v, pol_stream);
                     const unsigned long long e = ld_stream_u64(p.off + v + 1, pol_stream);
                     if (cur >= d) {  // not stale: d is still v's distance ("refined")
-                        degs[0] = (unsigned)(e - b);
-                        s_ebeg[tid] = b;
-                        s_d[tid] = (DistT)d;
-                        lives[0] = true;
+                        deg = (unsigned)(e - b);
+                        my_b = b;
+                        my_d = d;
+                        live = true;
                         if (p.dynamic) {  // work-waste signal: is this v's first expansion?
-                            const unsigned bit = 1u << (v & 31);
-                            fword[0] = atomicOr(p.expanded + (v >> 5), bit);  // result not waited for until the batch ends
-                            fbit[0] = bit;
+                            fbit = 1u << (v & 31);
+                            fword = atomicOr(p.expanded + (v >> 5), fbit);  // result not waited for until the batch ends
                         }
-                        if (p.split_deg && degs[0] > p.split_deg) degs[0] = spawn_chunks(p, v, d, b, degs[0], slot);
+                        if (p.split_deg && deg > p.split_deg) deg = spawn_chunks(p, v, d, b, deg, slot);
                     }
                 }
             }
-        }
-        unsigned deg = 0;
-        int live = 0;
-#pragma unroll
-        for (int r = 0; r < IPT; ++r) {
-            deg += degs[r];
-            live += lives[r] ? 1 : 0;
         }
         if (tid == 0) s_lnext = 0;
         if (prof) {
@@ -777,40 +766,54 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             s_prof[from_ring ? PR_N_RING : PR_N_LOCAL] += 1;
             t0 = t1;
         }
-        // exclusive scan of degrees over the CTA
+        // exclusive scan of degrees over the CTA, and the items with arcs compacted in
+        // scan order (rank r): s_scan[r] = first arc of item r in the batch's arc space,
+        // strictly increasing, with the sentinel s_scan[NZ] = E -- the owner search of the
+        // streaming loop relies on distinct starts (one bit per item start, below)
         unsigned x = deg;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
             const unsigned y = __shfl_up_sync(FULL, x, o);
             if (lane >= o) x += y;
         }
-        if (lane == 31) s_wsum[warp] = x;
-        int nlive = __syncthreads_count(live & 1);
-        if constexpr (IPT > 1) {
-#pragma unroll
-            for (int bit = 1; (1 << bit) <= IPT; ++bit) nlive += __syncthreads_count((live >> bit) & 1) << bit;
+        const unsigned nzm = __ballot_sync(FULL, deg > 0);
+        if (lane == 31) {
+            s_wsum[warp] = x;
+            s_wnz[warp] = __popc(nzm);
         }
+        const int nlive = __syncthreads_count(live);
         if (warp == 0) {
             const unsigned ws = lane < kWarps ? s_wsum[lane] : 0;
-            unsigned inc = ws;
+            const unsigned wn = lane < kWarps ? s_wnz[lane] : 0;
+            unsigned inc = ws, incn = wn;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
                 const unsigned y = __shfl_up_sync(FULL, inc, o);
-                if (lane >= o) inc += y;
+                const unsigned yn = __shfl_up_sync(FULL, incn, o);
+                if (lane >= o) {
+                    inc += y;
+                    incn += yn;
+                }
             }
-            if (lane < kWarps) s_wsum[lane] = inc - ws;
-            if (lane == kWarps - 1) s_E = inc;
+            if (lane < kWarps) {
+                s_wsum[lane] = inc - ws;
+                s_wnz[lane] = incn - wn;
+            }
+            if (lane == kWarps - 1) {
+                s_E = inc;
+                s_NZ = incn;
+                s_scan[incn] = inc;  // sentinel
+            }
         }
         __syncthreads();
-        {
-            unsigned ex = x - deg + s_wsum[warp];
-#pragma unroll
-            for (int r = 0; r < IPT; ++r) {
-                s_scan[tid * IPT + r] = ex;
-                ex += degs[r];
-            }
+        if (deg > 0) {
+            const unsigned r = s_wnz[warp] + __popc(nzm & lt_mask);
+            const unsigned ex = x - deg + s_wsum[warp];
+            s_scan[r] = ex;
+            s_eadj[r] = my_b - ex;  // arc e of the batch is adj[s_eadj[owner] + e]
+            s_d[r] = (DistT)my_d;
         }
-        const unsigned E = s_E;
+        const unsigned E = s_E, NZ = s_NZ;
         if (is_task) slot = s_slot;
         const int nexp = is_task ? 0 : nlive;  // a chunk is not a vertex expansion
         if (tid == 0) {
@@ -826,7 +829,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             tw = 0;
         }
 
-        __syncthreads();  // publishes s_scan / s_d / s_ebeg
+        __syncthreads();  // publishes s_scan / s_d / s_eadj
         if (CA && tid == 0) s_ahead = 0;  // every thread has read it (loop top)
         // ---------------------------------------------------- stream the batch's arcs
         // Warp w owns a contiguous slice of the batch's arc space and streams through
@@ -843,27 +846,37 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             const unsigned slice = (per + 31) / 32 * 32;  // small batches spread over many warps
             const unsigned wb = warp * slice;
             const unsigned we = (wb + slice) < E ? (wb + slice) : E;
-            // owner of each arc (largest i with scan[i] <= e, binary search in shared
-            // memory) and its coalesced {col, w} load
+            // Owner of each arc = the largest r with s_scan[r] <= e.  The warp walks its
+            // slice in windows of 32 consecutive arcs (one per lane) and carries `cur`, the
+            // owner of the window's first arc: lane l reads the start of item cur+1+l, the
+            // starts inside the window become one bit each (they are distinct), and an arc's
+            // owner is cur + the number of starts at or before it -- one shared load, one
+            // warp OR-reduction and a popcount per arc instead of a binary search
+            // (log2(BT) dependent shared loads per arc).  One binary search per slice.
+            unsigned cur = 0;
+            if (wb < we) {
+                unsigned lo = 0, hi = NZ - 1;
+                while (lo < hi) {
+                    const unsigned mid = (lo + hi + 1) >> 1;
+                    if (s_scan[mid] <= wb) lo = mid;
+                    else hi = mid - 1;
+                }
+                cur = lo;
+            }
             auto fetch = [&](unsigned base, unsigned (&own)[EPT], uint2 (&a)[EPT]) {
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {
-                    const unsigned e = base + j * 32 + lane;
-                    unsigned lo = 0, hi = got - 1;
-                    if (e < we) {
-                        while (lo < hi) {
-                            const unsigned mid = (lo + hi + 1) >> 1;
-                            if (s_scan[mid] <= e) lo = mid;
-                            else hi = mid - 1;
-                        }
-                    }
-                    own[j] = lo;
+                    const unsigned w0 = base + j * 32;
+                    const unsigned ix = cur + 1 + lane;
+                    const unsigned rel = s_scan[ix < NZ ? ix : NZ] - w0;  // >= 1 while w0 < E
+                    const unsigned bits = __reduce_or_sync(FULL, rel < 32u ? 1u << rel : 0u);
+                    own[j] = cur + __popc(bits & le_mask);
+                    cur += __popc(__ballot_sync(FULL, rel <= 32u));  // owner of the next window's first arc
                 }
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {  // EPT independent arc loads in flight
                     const unsigned e = base + j * 32 + lane;
-                    a[j] = e < we ? ld_stream_u2(p.adj + s_ebeg[own[j]] + (e - s_scan[own[j]]), pol_stream)
-                                  : make_uint2(0u, 0u);
+                    a[j] = e < we ? ld_stream_u2(p.adj + (s_eadj[own[j]] + e), pol_stream) : make_uint2(0u, 0u);
                 }
             };
             // head-bucket children stay on chip: first in this warp's own queue (warp-local
@@ -1151,7 +1164,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 unsigned long long idx = 0;
                 Head hd2;
                 bool tk;
-                const unsigned g = claim_batch<DistT, BT * IPT>(p, lane, sl, idx, hd2, st, tk);
+                const unsigned g = claim_batch<DistT, BT>(p, lane, sl, idx, hd2, st, tk);
                 if (lane == 0 && g) {
                     s_got = g;
                     s_slot = sl;
@@ -1227,9 +1240,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
 
         // ------------------------------------------------------------ complete
         // s_lnext final (also covers the E == 0 case); first expansions for the controller
-        int nfirst = 0;
-#pragma unroll
-        for (int r = 0; r < IPT; ++r) nfirst += __syncthreads_count(fbit[r] != 0 && (fword[r] & fbit[r]) == 0);
+        const int nfirst = __syncthreads_count(fbit != 0 && (fword & fbit) == 0);
         const unsigned kept = s_lnext < lcap ? s_lnext : lcap;
         const unsigned w_exp = s_wst[0], w_first = s_wst[1], w_kept = s_wst[4];
         if (tid == 0) {
