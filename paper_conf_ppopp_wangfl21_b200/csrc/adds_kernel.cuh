@@ -591,6 +591,12 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     unsigned* s_wqn = (unsigned*)(smem + L::o_wqn);
     __shared__ unsigned s_wst[5];  // warp-local continuation: expanded, first, edges, stale, kept
 
+    // staging: warp w owns s_items[w * kSeg, (w + 1) * kSeg) and its fill is a register;
+    // s_wcnt[w][o] = items warp w staged for bucket o (its ranks), turned into the warp's
+    // offset inside the CTA's reservation of bucket o at flush time
+    constexpr unsigned kSeg = (unsigned)kStage / kWarps;
+    static_assert(32 % kWarps == 0, "warps per CTA must divide 32");
+    __shared__ unsigned s_wcnt[kWarps][kMaxBuckets];
     __shared__ unsigned s_cnt[kMaxBuckets];
     __shared__ unsigned long long s_base[kMaxBuckets];
     __shared__ unsigned s_wsum[kWarps], s_wnz[kWarps];
@@ -610,6 +616,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     unsigned have_local = 0;  // uniform: items of the next batch already in s_lv/s_ld
 
     if (tid < (int)kMaxBuckets) s_cnt[tid] = 0;
+    for (int i = tid; i < kWarps * (int)kMaxBuckets; i += BT) (&s_wcnt[0][0])[i] = 0;
     if (tid < (int)kProfCounters) s_prof[tid] = 0;
     if (tid < 5) s_wst[tid] = 0;
     if (tid == 0) {
@@ -831,6 +838,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
 
         __syncthreads();  // publishes s_scan / s_d / s_eadj
         if (CA && tid == 0) s_ahead = 0;  // every thread has read it (loop top)
+        unsigned wfill = 0;  // warp-uniform: items staged in this warp's segment
         // ---------------------------------------------------- stream the batch's arcs
         // Warp w owns a contiguous slice of the batch's arc space and streams through
         // it with no CTA barrier (warps drift and keep the L1TEX queue busy); lanes
@@ -932,35 +940,34 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
                 return kept;
             };
-            // everything else: warp-aggregated staging for the CTA flush at batch end
-            // (or direct publication when the staging area is full)
+            // everything else: staged in the warp's own segment for the CTA flush at batch
+            // end (no shared atomics: the fill is a warp-uniform register and each bucket's
+            // count in s_wcnt[warp] is updated by one lane per bucket), or published
+            // directly when the segment is full
             auto emit = [&](const bool pg, const unsigned v, const unsigned long long ndv, const unsigned o) {
                 const unsigned act = __ballot_sync(FULL, pg);
                 if (!act) return;
-                // warp-aggregated staging slot for the CTA flush at batch end
-                const int leader = __ffs(act) - 1;
                 const unsigned nact = (unsigned)__popc(act);
-                unsigned pos = 0;
-                if (lane == leader) pos = atomicAdd(&s_total, nact);
-                pos = __shfl_sync(FULL, pos, leader);
-                if (pos + nact <= (unsigned)kStage) {
+                if (wfill + nact <= kSeg) {
                     if (pg) {
                         const unsigned peers = __match_any_sync(act, o);
                         const int pl = __ffs(peers) - 1;
                         unsigned r0 = 0;
-                        if (lane == pl) r0 = atomicAdd(&s_cnt[o], (unsigned)__popc(peers));
+                        if (lane == pl) {  // one lane per distinct bucket: no two lanes share the counter
+                            r0 = s_wcnt[warp][o];
+                            s_wcnt[warp][o] = r0 + (unsigned)__popc(peers);
+                        }
                         r0 = __shfl_sync(peers, r0, pl) + __popc(peers & lt_mask);
-                        const unsigned my = pos + __popc(act & lt_mask);
+                        const unsigned my = (unsigned)warp * kSeg + wfill + __popc(act & lt_mask);
                         s_items[my] = IT::make(v, ndv);
                         s_soff[my] = (unsigned char)o;
                         s_rank[my] = (unsigned short)r0;
                     }
+                    wfill += nact;
                 } else {
-                    // staging full (hubs): mark the slots this warp took as holes and
-                    // publish directly -- one reserve/avail pair per (warp, bucket)
+                    // segment full (hubs): publish directly -- one reserve/avail pair per
+                    // (warp, bucket)
                     if (pg) {
-                        const unsigned my = pos + __popc(act & lt_mask);
-                        if (my < (unsigned)kStage) s_soff[my] = 0xFF;
                         const unsigned peers = __match_any_sync(act, o);
                         const int pl = __ffs(peers) - 1;
                         const unsigned sl = (hs + o) & nbm;
@@ -994,11 +1001,20 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
 #pragma unroll
                 for (int j = 0; j < EPT; ++j)  // EPT independent L2 gathers in flight
-                    cur[j] = (nd[j] < kInf && !tiny)
-                                 ? (p.filt ? (DistT)min(filt_bound(ld_filt(p.filt + a[j].x), p.filt_shift),
-                                                        (unsigned long long)DistInf<DistT>::value)
-                                           : ld_keep(p.dist + a[j].x, pol_keep))
-                                 : (nd[j] < kInf ? DistInf<DistT>::value : (DistT)0);
+                    cur[j] = nd[j] < kInf ? DistInf<DistT>::value : (DistT)0;
+                if (!tiny) {
+                    if (p.filt == nullptr) {  // (uniform branch: the opt-in filter path stays out of the loop)
+#pragma unroll
+                        for (int j = 0; j < EPT; ++j)
+                            if (nd[j] < kInf) cur[j] = ld_keep(p.dist + a[j].x, pol_keep);
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < EPT; ++j)
+                            if (nd[j] < kInf)
+                                cur[j] = (DistT)min(filt_bound(ld_filt(p.filt + a[j].x), p.filt_shift),
+                                                    (unsigned long long)DistInf<DistT>::value);
+                    }
+                }
                 DistT old[EPT];
                 bool tried[EPT];
 #pragma unroll
@@ -1176,41 +1192,60 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
             }
         }
-        __syncthreads();
         {
-            const unsigned total = s_total < (unsigned)kStage ? s_total : (unsigned)kStage;
-            if (total > 0) {
+            const bool any_staged = __syncthreads_or(wfill != 0) != 0;
+            unsigned total = 0;
+            if (any_staged) {
                 // ---------------------------------------------------- flush to the ring
                 const long long tf = prof ? clock64() : 0;
-                if (warp == 0 && lane < (int)p.nb) {
-                    const unsigned c = s_cnt[lane];
-                    if (p.dynamic) {
-                        if (lane == 0) atomicAdd(&p.ctl->g_push, (unsigned long long)(total + s_direct));
-                        if (lane == (int)nbm && c) atomicAdd(&p.ctl->g_clip, (unsigned long long)c);
+                {
+                    // column scan of s_wcnt over the warps, all warps at once: lanes form
+                    // segments of kWarps (one per bucket), lane w%kWarps = warp w's count;
+                    // the segment's last lane holds the CTA's count for the bucket and
+                    // reserves it (returning atomic: the reserve, which also counts the
+                    // children for termination, precedes this CTA's completion release)
+                    constexpr unsigned kBPW = kWarps >= 32 ? 1u : 32u / kWarps;  // buckets per warp
+                    const unsigned o = (unsigned)warp * kBPW + (unsigned)lane / kWarps;
+                    const unsigned w = (unsigned)lane % kWarps;
+                    const bool mine = o < p.nb;
+                    const unsigned v = mine ? s_wcnt[w][o] : 0u;
+                    unsigned x = v;
+#pragma unroll
+                    for (unsigned d = 1; d < (unsigned)kWarps; d <<= 1) {
+                        const unsigned y = __shfl_up_sync(FULL, x, d, kWarps);
+                        if (w >= d) x += y;
                     }
-                    if (c) {
-                        const unsigned sl = (hs + lane) & nbm;
-                        // returning atomic: the reserve (which also counts the children for
-                        // termination) is performed before this CTA's completion atomic
-                        const unsigned long long b = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
-                        SSSP_FUZZ_AT(FZ_RESERVE);
-                        s_base[lane] = b;
-                        if (b + c > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
+                    if (mine) s_wcnt[w][o] = x - v;  // warp w's offset inside the CTA's reservation
+                    if (mine && w == (unsigned)kWarps - 1) {
+                        s_cnt[o] = x;
+                        if (x) {
+                            atomicAdd(&s_total, x);
+                            const unsigned long long b = atomicAdd(&p.bk[(hs + o) & nbm].reserve.v, (unsigned long long)x);
+                            SSSP_FUZZ_AT(FZ_RESERVE);
+                            s_base[o] = b;
+                            if (b + x > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
+                            if (p.dynamic && o == nbm) atomicAdd(&p.ctl->g_clip, (unsigned long long)x);
+                        }
                     }
                 }
                 __syncthreads();
-                for (unsigned i = tid; i < total; i += BT) {
-                    const unsigned o = s_soff[i];
-                    if (o == 0xFF) continue;  // hole left by a direct publication
+                total = s_total;
+                // each warp stores its own segment (coalesced runs per bucket)
+                for (unsigned i = lane; i < wfill; i += 32) {
+                    const unsigned my = (unsigned)warp * kSeg + i;
+                    const unsigned o = s_soff[my];
                     const unsigned sl = (hs + o) & nbm;
-                    const unsigned long long idx = s_base[o] + s_rank[i];
+                    const unsigned long long idx = s_base[o] + s_wcnt[warp][o] + s_rank[my];
                     SSSP_FUZZ_AT(FZ_PUBLISH);
                     // the slot's one writer this run (D13); beyond cap the run is aborted
-                    if (idx < p.cap) IT::store(p.ring + ((size_t)sl * p.cap + idx) * IT::kBytes, s_items[i]);
+                    if (idx < p.cap) IT::store(p.ring + ((size_t)sl * p.cap + idx) * IT::kBytes, s_items[my]);
                 }
+                __syncwarp();
+                if (lane < (int)p.nb) s_wcnt[warp][lane] = 0;  // this warp's row is no longer read
                 __syncthreads();
                 if (warp == 0 && lane < (int)p.nb) {
                     const unsigned c = s_cnt[lane];
+                    if (p.dynamic && lane == 0) atomicAdd(&p.ctl->g_push, (unsigned long long)(total + s_direct));
                     if (c) {
                         atomicAdd(&p.bk[(hs + lane) & nbm].avail.v, (unsigned long long)c);  // publish
                         s_cnt[lane] = 0;
