@@ -990,6 +990,15 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
             };
             // relax + push of one round whose arcs are loaded
+            // Relaxation write (A6).  With a gathered dist value cur (the plain L2 load that
+            // filters the atomics) the update is a fire-and-forget RED.min and the arc pushes
+            // iff nd < cur: whichever relaxation actually lowers dist[v] to x saw cur > x
+            // (dist only decreases), so every value dist[v] takes is pushed by its writer; a
+            // relaxation that lost a race to a smaller value pushes an item that is stale at
+            // its pop (skipped), or a duplicate of an equal one (expanded twice, same
+            // result).  Without the gather (tiny batches) or with the 16-bit filter (cur is
+            // only a bound) the returning atomicMin decides.
+            const bool fire = !tiny && p.filt == nullptr;
             auto body = [&](const unsigned base, const unsigned (&own)[EPT], const uint2 (&a)[EPT]) {
                 unsigned long long nd[EPT];
                 bool push[EPT];
@@ -1026,7 +1035,14 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         if (sum_unusable<kF>(nd[j], kInf)) {
                             if (!kF) atomicOr(&p.ctl->status, kStDistOverflow);  // 32-bit distances insufficient
                         } else if (nd[j] < (unsigned long long)cur[j]) {
-                            old[j] = atomic_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
+                            if (fire) {
+                                // fire-and-forget (D17): push on the gathered value; the RED
+                                // needs no round trip
+                                red_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
+                                old[j] = cur[j];
+                            } else {
+                                old[j] = atomic_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
+                            }
                             tried[j] = true;
                         }
                     }

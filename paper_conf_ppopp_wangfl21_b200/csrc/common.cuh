@@ -239,6 +239,14 @@ __device__ __forceinline__ unsigned long long atomic_min_keep(unsigned long long
     return r;
 }
 
+// fire-and-forget atomic min (RED: no result, no round trip for the issuing warp)
+__device__ __forceinline__ void red_min_keep(unsigned* a, unsigned v, unsigned long long pol) {
+    asm volatile("red.global.L2::cache_hint.min.u32 [%0], %1, %2;" ::"l"(a), "r"(v), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void red_min_keep(unsigned long long* a, unsigned long long v, unsigned long long pol) {
+    asm volatile("red.global.L2::cache_hint.min.u64 [%0], %1, %2;" ::"l"(a), "l"(v), "l"(pol) : "memory");
+}
+
 __device__ __forceinline__ unsigned long long globaltimer() {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
