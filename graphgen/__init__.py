@@ -177,12 +177,21 @@ CONFIGS = {
     "er": dict(kind="er", n=1 << 24, m=32 << 24, lo=1, hi=1 << 20, seed=4, source_seed=4),
     "batch": dict(kind="rmat", scale=24, edge_factor=16, lo=1, hi=255, seed=3, source_seed=5, k=512),
 }
+# Further families (not BASELINE configs): controller / launch-default validation on graphs
+# that sit on the other side of the defaults' average-degree switch (<= 8 arcs per vertex
+# selects the latency build) or change the weight range by orders of magnitude.
+EXTRA = {
+    "rmat_ef4": dict(kind="rmat", scale=24, edge_factor=4, lo=1, hi=255, seed=6, source_seed=6),
+    "er_d4": dict(kind="er", n=1 << 24, m=4 << 24, lo=1, hi=1 << 20, seed=7, source_seed=7),
+    "grid_wide": dict(kind="grid", W=4096, H=4096, lo=1, hi=1 << 20, seed=8, source_seed=8),
+    "rmat_wide": dict(kind="rmat", scale=24, edge_factor=16, lo=1, hi=1 << 20, seed=9, source_seed=9),
+}
 
 
 def make(config: str, scale_down: int = 0) -> CSR:
     """Build a named config graph.  ``scale_down`` shrinks it by 2^scale_down
     vertices (same recipe) for tests that must stay small."""
-    c = CONFIGS[config]
+    c = CONFIGS[config] if config in CONFIGS else EXTRA[config]
     if c["kind"] == "grid":
         W = max(2, c["W"] >> (scale_down // 2 + scale_down % 2))
         H = max(2, c["H"] >> (scale_down // 2))
@@ -196,7 +205,7 @@ def make(config: str, scale_down: int = 0) -> CSR:
 
 
 def config_sources(config: str, g: CSR, k: int = 1) -> np.ndarray:
-    c = CONFIGS[config]
+    c = CONFIGS[config] if config in CONFIGS else EXTRA[config]
     if "source" in c:
         return np.array([c["source"]] * k, dtype=np.uint32)[:k]
     return sources(g, k, c["source_seed"])

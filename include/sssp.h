@@ -207,9 +207,11 @@ typedef struct sssp_trace_entry {
     uint32_t active;         /* active buckets after the step */
     uint32_t waste_permille; /* re-expansion share of recent expansions (work-waste signal) */
     uint32_t reason;         /* bits 0-7: 1 = head-bucket switch, 2 = periodic controller step;
-                                bits 8+: decision inputs (1 low util, 2 high util, 4 work beyond the
+                                bits 8-16: decision inputs (1 low util, 2 high util, 4 work beyond the
                                 window, 8 wasteful, 16 frugal, 32 clipping, 64 waste known,
-                                128 start-up over, 256 settled) */
+                                128 start-up over, 256 settled);
+                                bits 20-29: share of recent pushes clipped into the tail (permille),
+                                bit 30: that share is measured (>= 64K recent pushes) */
 } sssp_trace_entry;
 
 /* Opaque handle: owns the device CSR, the workspace (bucket ring, counters,

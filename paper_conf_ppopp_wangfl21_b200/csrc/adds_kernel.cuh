@@ -100,8 +100,7 @@ __device__ __forceinline__ long long warp_sum_s64(long long x) {
 // window (utilisation = window items x average degree vs resident threads,
 // P:211) and the tail (clip share); plus the recent re-expansion
 // share of expansions (work-waste signal, R6).  Readings:
-//   clip   tail >= clip_pct of all pending, or >= 1/2 of recent pushes were
-//          clipped into the tail (2 steps apart)  -> Delta x2, floor = Delta
+//   clip   tail >= clip_pct of all pending (2 steps apart) -> Delta x2, floor = Delta
 //   waste  share > waste_hi after settling        -> Delta /2 (not below floor)
 //   grow   window under-utilised AND share < lo   -> Delta x2
 //   A      active buckets follow the same two signals one step at a time
@@ -151,7 +150,13 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
     constexpr unsigned ratio_gate = 250u;
     const bool frugal = (!waste_known || waste < p.waste_lo) &&
                         (ratio_x100 < ratio_gate || !waste_known || waste * 2 < p.waste_lo) && progressed;
-    const bool clipping = (total >= 64 && tail * 100 >= (long long)p.clip_pct * total) || (clip_known && clip >= 500);
+    // the paper's rule only: the share of recent pushes clipped into the tail is
+    // recorded in the trace but does not decide -- early in a run most pushes carry large
+    // tentative distances, and reacting to them grew ER from its best Delta (2^15) to 2^16
+    // (work 1.01x -> 1.17x, profiles/r02_sweeps.md §3)
+    (void)clip;
+    (void)clip_known;
+    const bool clipping = total >= 64 && tail * 100 >= (long long)p.clip_pct * total;
     // settled: enough steps AND the head has switched twice since the last
     // change, so the ring has turned over and the items placed under the previous
     // Delta -- whose slots now mix priorities -- are no longer what the
@@ -233,7 +238,7 @@ __device__ __forceinline__ unsigned recent_clip(const Params<DistT>& p, bool& kn
 template <typename DistT>
 __device__ void commit_step(const Params<DistT>& p, const Head hd, const Head nhd, bool kchanged, unsigned since,
                             long long total, long long win, long long tail, unsigned waste, unsigned reason,
-                            unsigned flags) {
+                            unsigned flags, unsigned clip, bool clip_known) {
     Head seen;
     if (!cas_head(&p.ctl->head, hd, nhd, seen)) return;
     if (reason == 1) atomicAdd(&p.ctl->head_switches, 1u);
@@ -261,7 +266,8 @@ __device__ void commit_step(const Params<DistT>& p, const Head hd, const Head nh
             e.delta_log2 = meta_k(nhd.meta);
             e.active = meta_A(nhd.meta);
             e.waste_permille = waste;
-            e.reason = reason | (flags << 8);
+            e.reason = reason | ((flags & 0x1ffu) << 8) | ((clip < 1000u ? clip : 1000u) << 20) |
+                       (clip_known ? 1u << 30 : 0u);
             p.trace[t] = e;
         }
     }
@@ -308,7 +314,7 @@ __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lan
     const Head nhd{rehead(hd.h + o, k, d.k),
                    pack_meta((hs + o) & (nb - 1), d.k, d.A, d.flo, d.since, d.ceil)};
     SSSP_FUZZ_AT(FZ_HEAD);
-    commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 1u, d.flags);
+    commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 1u, d.flags, clip, cknown);
     return false;
 }
 
@@ -332,7 +338,7 @@ __device__ void periodic_step(const Params<DistT>& p, const int lane) {
                                  ld_relaxed_u64(&p.ctl->g_first) >= p.startup_first ||
                                      ld_relaxed_u32(&p.ctl->head_switches) >= 32u);
     const Head nhd{rehead(hd.h, k, d.k), pack_meta(hs, d.k, d.A, d.flo, d.since, d.ceil)};
-    commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 2u, d.flags);
+    commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 2u, d.flags, clip, cknown);
 }
 
 // --------------------------------------------------------------- weight arithmetic
@@ -940,54 +946,91 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
                 return kept;
             };
+            // A full segment is published by its warp alone (warp_flush): one reserve and one
+            // avail atomic per bucket present, coalesced stores -- 32x fewer round trips than
+            // publishing each push directly.  The children are counted (reserve) before this
+            // batch's completion, as at the CTA flush.
+            auto warp_flush = [&]() {
+                const unsigned c = lane < (int)p.nb ? s_wcnt[warp][lane] : 0u;
+                const unsigned sl = (hs + (unsigned)lane) & nbm;
+                unsigned long long b = 0;
+                if (c) {
+                    b = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
+                    SSSP_FUZZ_AT(FZ_RESERVE);
+                    if (b + c > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
+                    if (p.dynamic && lane == (int)nbm) atomicAdd(&p.ctl->g_clip, (unsigned long long)c);
+                }
+                for (unsigned i0 = 0; i0 < wfill; i0 += 32) {
+                    const unsigned i = i0 + (unsigned)lane;
+                    const unsigned my = (unsigned)warp * kSeg + i;
+                    const unsigned o = i < wfill ? s_soff[my] : 0u;
+                    const unsigned long long bo = __shfl_sync(FULL, b, (int)o);
+                    if (i < wfill) {
+                        const unsigned long long idx = bo + s_rank[my];
+                        SSSP_FUZZ_AT(FZ_PUBLISH);
+                        // the slot's one writer this run (D13); beyond cap the run is aborted
+                        if (idx < p.cap) IT::store(p.ring + ((size_t)((hs + o) & nbm) * p.cap + idx) * IT::kBytes, s_items[my]);
+                    }
+                }
+                __syncwarp();
+                if (c) atomicAdd(&p.bk[sl].avail.v, (unsigned long long)c);  // publish
+                if (lane < (int)p.nb) s_wcnt[warp][lane] = 0;
+                if (lane == 0) atomicAdd(&s_direct, wfill);
+                wfill = 0;
+                __syncwarp();
+            };
             // everything else: staged in the warp's own segment for the CTA flush at batch
             // end (no shared atomics: the fill is a warp-uniform register and each bucket's
-            // count in s_wcnt[warp] is updated by one lane per bucket), or published
-            // directly when the segment is full
+            // count in s_wcnt[warp] is updated by one lane per bucket)
             auto emit = [&](const bool pg, const unsigned v, const unsigned long long ndv, const unsigned o) {
                 const unsigned act = __ballot_sync(FULL, pg);
                 if (!act) return;
                 const unsigned nact = (unsigned)__popc(act);
-                if (wfill + nact <= kSeg) {
-                    if (pg) {
-                        const unsigned peers = __match_any_sync(act, o);
-                        const int pl = __ffs(peers) - 1;
-                        unsigned r0 = 0;
-                        if (lane == pl) {  // one lane per distinct bucket: no two lanes share the counter
-                            r0 = s_wcnt[warp][o];
-                            s_wcnt[warp][o] = r0 + (unsigned)__popc(peers);
+                if (wfill + nact > kSeg) {
+                    if constexpr (WLC) {
+                        // latency build: segments rarely fill; publish just these pushes
+                        // (keeps the warp-local hop loop short, ROAD 33.8 vs 32.2 ms with
+                        // warp_flush here)
+                        if (pg) {
+                            const unsigned peers = __match_any_sync(act, o);
+                            const int pl = __ffs(peers) - 1;
+                            const unsigned sl = (hs + o) & nbm;
+                            unsigned long long b0 = 0;
+                            if (lane == pl) {
+                                const unsigned c = (unsigned)__popc(peers);
+                                b0 = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
+                                if (b0 + c > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
+                                atomicAdd(&s_direct, c);
+                                SSSP_FUZZ_AT(FZ_RESERVE);
+                            }
+                            b0 = __shfl_sync(peers, b0, pl);
+                            const unsigned long long idx = b0 + __popc(peers & lt_mask);
+                            // the slot's one writer this run (D13); beyond cap the run is aborted
+                            if (idx < p.cap) IT::store(p.ring + ((size_t)sl * p.cap + idx) * IT::kBytes, IT::make(v, ndv));
+                            SSSP_FUZZ_AT(FZ_PUBLISH);
+                            __syncwarp(peers);
+                            if (lane == pl) atomicAdd(&p.bk[sl].avail.v, (unsigned long long)__popc(peers));
                         }
-                        r0 = __shfl_sync(peers, r0, pl) + __popc(peers & lt_mask);
-                        const unsigned my = (unsigned)warp * kSeg + wfill + __popc(act & lt_mask);
-                        s_items[my] = IT::make(v, ndv);
-                        s_soff[my] = (unsigned char)o;
-                        s_rank[my] = (unsigned short)r0;
-                    }
-                    wfill += nact;
-                } else {
-                    // segment full (hubs): publish directly -- one reserve/avail pair per
-                    // (warp, bucket)
-                    if (pg) {
-                        const unsigned peers = __match_any_sync(act, o);
-                        const int pl = __ffs(peers) - 1;
-                        const unsigned sl = (hs + o) & nbm;
-                        unsigned long long b0 = 0;
-                        if (lane == pl) {
-                            const unsigned c = (unsigned)__popc(peers);
-                            b0 = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
-                            if (b0 + c > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
-                            atomicAdd(&s_direct, c);
-                            SSSP_FUZZ_AT(FZ_RESERVE);
-                        }
-                        b0 = __shfl_sync(peers, b0, pl);
-                        const unsigned long long idx = b0 + __popc(peers & lt_mask);
-                        // the slot's one writer this run (D13); beyond cap the run is aborted
-                        if (idx < p.cap) IT::store(p.ring + ((size_t)sl * p.cap + idx) * IT::kBytes, IT::make(v, ndv));
-                        SSSP_FUZZ_AT(FZ_PUBLISH);
-                        __syncwarp(peers);
-                        if (lane == pl) atomicAdd(&p.bk[sl].avail.v, (unsigned long long)__popc(peers));
+                        return;
+                    } else {
+                        warp_flush();
                     }
                 }
+                if (pg) {
+                    const unsigned peers = __match_any_sync(act, o);
+                    const int pl = __ffs(peers) - 1;
+                    unsigned r0 = 0;
+                    if (lane == pl) {  // one lane per distinct bucket: no two lanes share the counter
+                        r0 = s_wcnt[warp][o];
+                        s_wcnt[warp][o] = r0 + (unsigned)__popc(peers);
+                    }
+                    r0 = __shfl_sync(peers, r0, pl) + __popc(peers & lt_mask);
+                    const unsigned my = (unsigned)warp * kSeg + wfill + __popc(act & lt_mask);
+                    s_items[my] = IT::make(v, ndv);
+                    s_soff[my] = (unsigned char)o;
+                    s_rank[my] = (unsigned short)r0;
+                }
+                wfill += nact;
             };
             // relax + push of one round whose arcs are loaded
             // Relaxation write (A6).  With a gathered dist value cur (the plain L2 load that

@@ -25,6 +25,7 @@ def main():
     ap.add_argument("--deltas", default="", help="comma list of log2 Delta for static sweeps")
     ap.add_argument("--extra", default="{}", help="JSON dict merged into every static set")
     ap.add_argument("--profile", action="store_true", help="add SSSP_FLAG_PROFILE and print phase fractions")
+    ap.add_argument("--variant", default="", help="library build: loads libsssp_<variant>.so")
     a = ap.parse_args()
     import torch
     g = gg.make(a.config, scale_down=a.scale_down)
@@ -33,7 +34,7 @@ def main():
     extra = json.loads(a.extra)
     for k in [int(x) for x in a.deltas.split(",") if x]:
         sets.append(dict(delta_mode=1, delta_init=1 << k, **extra))
-    G = sssp.Graph.from_csr(g)
+    G = sssp.Graph.from_csr(g, variant=a.variant)
     base = sssp.sssp_options_default()
     out = torch.empty(g.n, dtype=torch.int64, device="cuda")
     for s in sets:
