@@ -950,7 +950,29 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             // avail atomic per bucket present, coalesced stores -- 32x fewer round trips than
             // publishing each push directly.  The children are counted (reserve) before this
             // batch's completion, as at the CTA flush.
+            // Rank the warp's staged items within their buckets (s_rank) and count them per
+            // bucket (s_wcnt[warp]): deferred from the push sites to here, where a warp-wide
+            // match_any covers 32 staged items instead of the one or two pushes of a site.
+            auto rank_segment = [&]() {
+                for (unsigned i0 = 0; i0 < wfill; i0 += 32) {
+                    const unsigned i = i0 + (unsigned)lane;
+                    const unsigned my = (unsigned)warp * kSeg + i;
+                    const bool valid = i < wfill;
+                    const unsigned o = valid ? s_soff[my] : 0xFFu;
+                    const unsigned peers = __match_any_sync(FULL, o);
+                    const int pl = __ffs(peers) - 1;
+                    unsigned r0 = 0;
+                    if (valid && lane == pl) {  // one lane per distinct bucket
+                        r0 = s_wcnt[warp][o];
+                        s_wcnt[warp][o] = r0 + (unsigned)__popc(peers);
+                    }
+                    r0 = __shfl_sync(FULL, r0, pl) + __popc(peers & lt_mask);
+                    if (valid) s_rank[my] = (unsigned short)r0;
+                    __syncwarp();
+                }
+            };
             auto warp_flush = [&]() {
+                rank_segment();
                 const unsigned c = lane < (int)p.nb ? s_wcnt[warp][lane] : 0u;
                 const unsigned sl = (hs + (unsigned)lane) & nbm;
                 unsigned long long b = 0;
@@ -980,8 +1002,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 __syncwarp();
             };
             // everything else: staged in the warp's own segment for the CTA flush at batch
-            // end (no shared atomics: the fill is a warp-uniform register and each bucket's
-            // count in s_wcnt[warp] is updated by one lane per bucket)
+            // end (no shared atomics: the fill is a warp-uniform register; bucket ranks and
+            // counts are computed at flush time)
             auto emit = [&](const bool pg, const unsigned v, const unsigned long long ndv, const unsigned o) {
                 const unsigned act = __ballot_sync(FULL, pg);
                 if (!act) return;
@@ -1016,19 +1038,10 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         warp_flush();
                     }
                 }
-                if (pg) {
-                    const unsigned peers = __match_any_sync(act, o);
-                    const int pl = __ffs(peers) - 1;
-                    unsigned r0 = 0;
-                    if (lane == pl) {  // one lane per distinct bucket: no two lanes share the counter
-                        r0 = s_wcnt[warp][o];
-                        s_wcnt[warp][o] = r0 + (unsigned)__popc(peers);
-                    }
-                    r0 = __shfl_sync(peers, r0, pl) + __popc(peers & lt_mask);
+                if (pg) {  // (bucket ranks are assigned at flush time, rank_segment)
                     const unsigned my = (unsigned)warp * kSeg + wfill + __popc(act & lt_mask);
                     s_items[my] = IT::make(v, ndv);
                     s_soff[my] = (unsigned char)o;
-                    s_rank[my] = (unsigned short)r0;
                 }
                 wfill += nact;
             };
@@ -1230,6 +1243,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 const unsigned nf = (unsigned)__popc(__ballot_sync(FULL, fbit != 0 && (fword & fbit) == 0));
                 if (lane == 0 && nf) atomicAdd(&s_wst[1], nf);
             }
+            rank_segment();  // bucket ranks of this warp's staged pushes, before the CTA flush
         }
         if constexpr (CA) {
             // the batch's claim state (s_got/s_slot/s_idx/s_head/s_task) was consumed before
