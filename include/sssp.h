@@ -81,8 +81,10 @@ typedef enum sssp_status {
                                          renumbered by descending in-degree inside the library; inputs and
                                          outputs stay in the caller's numbering; D15) */
 #define SSSP_FLAG_NO_RELABEL 0x800u   /* never relabel (default: relabel when max in-degree > 64 x average) */
-#define SSSP_FLAG_ADAPT_ACTIVE 0x40u  /* let the controller vary the number of active buckets;
-                                        off by default: on our workloads it raised re-expansions */
+#define SSSP_FLAG_ADAPT_ACTIVE 0x40u  /* (the default since round 2; kept for source compatibility) the
+                                        controller varies the number of active buckets between
+                                        the degree-based default A0 and 2*A0 from the CTAs holding work */
+#define SSSP_FLAG_FIXED_ACTIVE 0x1000u /* ablation: keep the active-bucket count at its initial value */
 #define SSSP_FLAG_L2_PERSIST 0x20u /* reserve the L2 persisting set-aside for dist (raises the device-wide
                                      cudaLimitPersistingL2CacheSize to min(dist bytes, maximum)) and mark
                                      dist accesses evict_last.  Off by default: measured on B200
@@ -204,7 +206,9 @@ typedef struct sssp_trace_entry {
     uint64_t pending_window; /* same, active buckets only */
     uint64_t pending_tail;   /* same, tail (clip) bucket */
     uint32_t delta_log2;     /* Delta in force after the step */
-    uint32_t active;         /* active buckets after the step */
+    uint32_t active;         /* bits 0-7: active buckets after the step; bits 8-15: floor of log2 Delta
+                                (the clip bound); bits 16-23: ceiling of log2 Delta (a value
+                                measured wasteful, not grown into again; 255 = none) */
     uint32_t waste_permille; /* re-expansion share of recent expansions (work-waste signal) */
     uint32_t reason;         /* bits 0-7: 1 = head-bucket switch, 2 = periodic controller step;
                                 bits 8-16: decision inputs (1 low util, 2 high util, 4 work beyond the

@@ -60,7 +60,9 @@ struct Params {
     unsigned nb;               // ring buckets, power of two <= 32
     unsigned long long cap;    // items per bucket array, power of two
     unsigned dynamic;          // Delta controller enabled
-    unsigned adapt_active;     // controller may vary the active-bucket count
+    unsigned adapt_active;     // controller varies the active-bucket count in [a_min, a_max]
+    unsigned a_min, a_max;
+    unsigned grid;             // CTAs of this launch (utilisation = CTAs holding a batch)
     unsigned clip_pct;         // P:207 (65)
     unsigned settle;           // P:215 head switches between Delta changes
     unsigned util_lo_pct, util_hi_pct;  // P:211 limits, % of resident threads
@@ -121,7 +123,7 @@ template <typename DistT>
 __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, unsigned flo, unsigned since,
                               unsigned ceil, bool head_switch, long long total, long long tail, long long win, unsigned waste,
                               bool waste_known, unsigned clip, bool clip_known, unsigned ratio_x100,
-                              bool progressed) {
+                              bool progressed, long long busy) {
     // since = [0,8) controller steps, [8,16) head switches since the last change
     unsigned steps = since & 0xffu, hsw = (since >> 8) & 0xffu;
     steps = steps < 255u ? steps + 1 : 255u;
@@ -185,14 +187,17 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
         d.changed = true;
     }
     if (d.changed) d.since = 0;
-    // fine-grained knob: one more active bucket only when the hardware is
-    // under-utilised, work waits beyond the window and almost nothing is
-    // re-expanded; back to fewer when wasteful or busy
+    // fine-grained knob: utilisation as the paper measures it -- the work
+    // assigned, here the CTAs holding a batch.  One more active bucket while CTAs are idle,
+    // work waits beyond the window and re-expansion is low; one fewer when every CTA is
+    // busy or the run is wasteful.  Bounded to [a_min, a_max] around the degree-based
+    // default (a wider window on road-like graphs fed the Delta shrink spiral, sweeps r01 §26)
     if (p.adapt_active) {
-        if (low && beyond && waste_known && waste < p.waste_lo / 4 && ratio_x100 < 115 && steps >= p.settle &&
-            A < p.nb)
+        const bool idle_ctas = busy * 10 < (long long)p.grid * 9;
+        const bool all_busy = busy >= (long long)p.grid;
+        if (idle_ctas && beyond && frugal && A < p.a_max)
             d.A = A + 1;
-        else if ((wasteful || high) && A > 1)
+        else if ((wasteful || all_busy) && A > p.a_min)
             d.A = A - 1;
     }
     return d;
@@ -264,7 +269,7 @@ __device__ void commit_step(const Params<DistT>& p, const Head hd, const Head nh
             e.pending_window = (unsigned long long)win;
             e.pending_tail = (unsigned long long)tail;
             e.delta_log2 = meta_k(nhd.meta);
-            e.active = meta_A(nhd.meta);
+            e.active = meta_A(nhd.meta) | (meta_floor(nhd.meta) << 8) | (meta_ceil(nhd.meta) << 16);
             e.waste_permille = waste;
             e.reason = reason | ((flags & 0x1ffu) << 8) | ((clip < 1000u ? clip : 1000u) << 20) |
                        (clip_known ? 1u << 30 : 0u);
@@ -310,7 +315,8 @@ __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lan
     const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), meta_ceil(hd.meta), true, total, tail, win, waste,
                                  known, clip, cknown, cumulative_ratio(p),
                                  ld_relaxed_u64(&p.ctl->g_first) >= p.startup_first ||
-                                     ld_relaxed_u32(&p.ctl->head_switches) >= 32u);
+                                     ld_relaxed_u32(&p.ctl->head_switches) >= 32u,
+                                 (long long)ld_relaxed_u64(&p.ctl->g_busy));
     const Head nhd{rehead(hd.h + o, k, d.k),
                    pack_meta((hs + o) & (nb - 1), d.k, d.A, d.flo, d.since, d.ceil)};
     SSSP_FUZZ_AT(FZ_HEAD);
@@ -336,7 +342,8 @@ __device__ void periodic_step(const Params<DistT>& p, const int lane) {
     const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), meta_ceil(hd.meta), false, total, tail, win, waste,
                                  known, clip, cknown, cumulative_ratio(p),
                                  ld_relaxed_u64(&p.ctl->g_first) >= p.startup_first ||
-                                     ld_relaxed_u32(&p.ctl->head_switches) >= 32u);
+                                     ld_relaxed_u32(&p.ctl->head_switches) >= 32u,
+                                 (long long)ld_relaxed_u64(&p.ctl->g_busy));
     const Head nhd{rehead(hd.h, k, d.k), pack_meta(hs, d.k, d.A, d.flo, d.since, d.ceil)};
     commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 2u, d.flags, clip, cknown);
 }
@@ -619,6 +626,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     const unsigned local_max = p.local_max < (unsigned)BT ? p.local_max : (unsigned)BT;
     unsigned long long c_vert = 0, c_edges = 0, c_push = 0, c_stale = 0, c_local = 0;  // thread 0
     unsigned backoff = 0;
+    const bool track_busy = p.dynamic && p.adapt_active;
+    bool busy_cta = false;  // warp 0 lane 0: this CTA is counted in g_busy
     unsigned have_local = 0;  // uniform: items of the next batch already in s_lv/s_ld
 
     if (tid < (int)kMaxBuckets) s_cnt[tid] = 0;
@@ -665,6 +674,10 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 } else if (g) {
                     cmd = CMD_WORK;
                     if (lane == 0) {
+                        if (track_busy && !busy_cta) {  // idle -> holding work (utilisation)
+                            red_add_u64(&p.ctl->g_busy, 1ull);
+                            busy_cta = true;
+                        }
                         s_got = g;
                         s_slot = sl;
                         s_idx = idx;
@@ -676,6 +689,10 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     if (try_advance<DistT>(p, hd, lane)) {
                         cmd = CMD_EXIT;
                     } else if (lane == 0) {
+                        if (track_busy && busy_cta) {  // found nothing to claim: idle
+                            red_add_u64(&p.ctl->g_busy, ~0ull);
+                            busy_cta = false;
+                        }
                         if (globaltimer() - p.ctl->t_start > p.timeout_ns) atomicOr(&p.ctl->status, kStTimeout);
                         backoff = backoff ? (backoff * 2 < p.max_backoff_ns ? backoff * 2 : p.max_backoff_ns) : 32;
                         __nanosleep(backoff);

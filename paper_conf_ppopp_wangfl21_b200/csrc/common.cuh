@@ -121,6 +121,8 @@ struct alignas(128) Ctl {
     char pad7_[120];
     unsigned long long g_clip;    // items pushed into the tail bucket (clipped)
     char pad8_[120];
+    unsigned long long g_busy;    // CTAs holding a batch (the paper's "work assigned")
+    char pad9_[120];
     unsigned long long st_local;  // items continued CTA-locally
     // statistics (flushed once per CTA at exit, or by finalize)
     unsigned long long st_vertices, st_edges, st_pushes, st_stale;
@@ -259,6 +261,9 @@ __device__ __forceinline__ unsigned long long globaltimer() {
 // increment (try_advance / bucket_pending read `done` with ld.acquire before
 // `reserve` and `local`), so a bucket can never look complete while one of its
 // items' children is not yet counted (exact termination).
+__device__ __forceinline__ void red_add_u64(unsigned long long* p, unsigned long long v) {
+    asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 __device__ __forceinline__ void red_release_add_u64(unsigned long long* p, unsigned long long v) {
     asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }

@@ -318,7 +318,9 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
     p.nb = g->opts.num_buckets;
     p.cap = w.cap;
     p.dynamic = g->opts.delta_mode == SSSP_DELTA_DYNAMIC;
-    p.adapt_active = (g->opts.flags & SSSP_FLAG_ADAPT_ACTIVE) ? 1u : 0u;
+    // active buckets adapt by default; SSSP_FLAG_FIXED_ACTIVE pins them at active_init
+    p.adapt_active = (g->opts.flags & SSSP_FLAG_FIXED_ACTIVE) ? 0u : 1u;
+    p.grid = grid;
     p.clip_pct = g->opts.clip_pct;
     p.settle = g->opts.settle_head_switches;
     p.util_lo_pct = g->opts.util_lo_pct;
@@ -434,6 +436,8 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     const unsigned span = kF ? heuristic_k(g) : g->heur_k_span;
     Head h0{0ull, pack_meta(0, k, A0, std::min(k, span), 0)};
     Params<DistT> p = make_params<DistT>(g, w, grid, bt, k_max, conc);
+    p.a_min = A0;
+    p.a_max = std::min(g->opts.num_buckets, std::max(2u, 2u * A0));
 
     const unsigned aux_grid = (unsigned)g->sm_count * 8 / conc + 1;
     CK(cudaEventRecord(w.ev[0], s), "event");

@@ -276,26 +276,56 @@ def test_async_flag_and_stats():
     assert np.array_equal(sssp.to_u64(out), oracle.dijkstra(g, s)[0])
 
 
-def test_trace_invariants():
-    g = gg.make("rmat", scale_down=6)
-    s = int(gg.config_sources("rmat", g, 1)[0])
-    G = sssp.Graph.from_csr(g, flags=sssp.SSSP_FLAG_TRACE)
-    d = sssp.to_u64(G.run(s))
-    assert np.array_equal(d, oracle.dijkstra(g, s)[0])
-    st = G.stats()
-    tr = G.trace()
+def check_controller_trace(tr, st, a_lo, a_hi):
+    """The Delta controller's invariants from its committed steps."""
     assert sum(1 for e in tr if e["reason"] & 255 == 1) == min(st["head_switches"], 65536)
+    prev_flo = 0
     for e in tr:
+        A, flo, ceil = e["active"] & 255, (e["active"] >> 8) & 255, (e["active"] >> 16) & 255
         assert e["reason"] & 255 in (1, 2)
-        assert 1 <= e["active"] <= 32
+        assert a_lo <= A <= a_hi                      # P:217 knob within its bounds
         assert 0 <= e["delta_log2"] <= 31
+        assert e["delta_log2"] >= flo                 # never below the clip bound (P:207)
+        assert flo >= prev_flo                        # the bound only rises (on clip steps)
+        prev_flo = flo
+        assert ceil == 255 or ceil > e["delta_log2"]  # a ceiling is a Delta measured wasteful, above k
         assert e["waste_permille"] <= 1000
         assert e["pending_tail"] <= e["pending_total"] and e["pending_window"] <= e["pending_total"]
-    # Delta moves one power of two per step and only after settling, except clip steps
+    # Delta moves one power of two per step; a change that is not a clip step needs the ring
+    # to have turned over: >= 2 head switches since the previous change (P:215, reading R7)
     ks = [e["delta_log2"] for e in tr]
     assert all(abs(a - b) <= 1 for a, b in zip(ks, ks[1:]))
+    last_change, switches = None, 0
+    for i in range(1, len(tr)):
+        if tr[i]["reason"] & 255 == 1:
+            switches += 1
+        if ks[i] != ks[i - 1]:
+            clip_step = (tr[i]["reason"] >> 8) & 32
+            if not clip_step and last_change is not None:
+                assert switches >= 2, (i, switches)
+            last_change, switches = i, 0
     ts = [e["time_ns"] for e in tr]
     assert len(tr) < 2 or max(ts) >= min(ts)
+
+
+@pytest.mark.parametrize("config,a_lo,a_hi", [("rmat", 4, 8), ("road", 1, 2), ("er", 4, 8)])
+def test_trace_invariants(config, a_lo, a_hi):
+    g = gg.make(config, scale_down=6)
+    for s in gg.config_sources(config, g, 3):
+        G = sssp.Graph.from_csr(g, flags=sssp.SSSP_FLAG_TRACE)
+        d = sssp.to_u64(G.run(int(s)))
+        assert np.array_equal(d, oracle.dijkstra(g, int(s))[0])
+        check_controller_trace(G.trace(), G.stats(), a_lo, a_hi)
+        G.close()
+
+
+def test_trace_invariants_full_size_road():
+    """ROAD at full size: ~300 head switches, the controller's longest run here."""
+    g = gg.make("road")
+    s = int(gg.config_sources("road", g, 1)[0])
+    G = sssp.Graph.from_csr(g, flags=sssp.SSSP_FLAG_TRACE)
+    G.run(s)
+    check_controller_trace(G.trace(), G.stats(), 1, 2)
 
 
 def test_repeat_runs_deterministic_and_reusable():

@@ -41,11 +41,12 @@ def main():
     if a.changes:
         keep = {0}
         for i in range(1, len(tr)):
-            if (tr[i]["delta_log2"], tr[i]["active"]) != (tr[i - 1]["delta_log2"], tr[i - 1]["active"]):
+            if (tr[i]["delta_log2"], tr[i]["active"] & 255) != (tr[i - 1]["delta_log2"], tr[i - 1]["active"] & 255):
                 keep.update({i - 1, i})
         rows = [tr[i] for i in sorted(keep | set(range(0, len(tr), step)))]
     for e in rows:
-        print(f'{(e["time_ns"] - t0) / 1e3:9.1f}us head={e["head"]:8d} k={e["delta_log2"]:2d} A={e["active"]:2d} '
+        print(f'{(e["time_ns"] - t0) / 1e3:9.1f}us head={e["head"]:8d} k={e["delta_log2"]:2d} A={e["active"] & 255:2d} '
+              f'flo={(e["active"] >> 8) & 255:2d} '
               f'pend={e["pending_total"]:9d} win={e["pending_window"]:9d} tail={e["pending_tail"]:8d} '
               f'waste={e["waste_permille"]:4d} clip={(e["reason"] >> 20) & 1023:4d}{"*" if e["reason"] >> 30 & 1 else " "} '
               f'why={e["reason"] & 255} flags={(e["reason"] >> 8) & 511:09b}')
