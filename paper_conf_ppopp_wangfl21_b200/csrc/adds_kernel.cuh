@@ -152,13 +152,13 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
     constexpr unsigned ratio_gate = 250u;
     const bool frugal = (!waste_known || waste < p.waste_lo) &&
                         (ratio_x100 < ratio_gate || !waste_known || waste * 2 < p.waste_lo) && progressed;
-    // the paper's rule only: the share of recent pushes clipped into the tail is
-    // recorded in the trace but does not decide -- early in a run most pushes carry large
-    // tentative distances, and reacting to them grew ER from its best Delta (2^15) to 2^16
-    // (work 1.01x -> 1.17x, profiles/r02_sweeps.md §3)
-    (void)clip;
-    (void)clip_known;
-    const bool clipping = total >= 64 && tail * 100 >= (long long)p.clip_pct * total;
+    // the paper's rule -- the tail holds >= 65 % of the pending items -- applied to
+    // live clipping: recent pushes must still be landing in the tail (>= 10 %) and enough work
+    // must be pending to matter.  On its own the push share fired on the large tentative
+    // distances early in a run (ER grown from its best Delta 2^15 to 2^16, work 1.01x -> 1.17x)
+    // and the pending share on a drained ring whose last items sat in the tail slot (ER with
+    // degree 4 doubled Delta from 2^21 to 2^31 in its drain; profiles/r02_sweeps.md §5, §7)
+    const bool clipping = total >= 1024 && tail * 100 >= (long long)p.clip_pct * total && clip_known && clip >= 100;
     // settled: enough steps AND the head has switched twice since the last
     // change, so the ring has turned over and the items placed under the previous
     // Delta -- whose slots now mix priorities -- are no longer what the
@@ -171,6 +171,13 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
         d.k = k + 1;  // clipping: raise Delta and its lower bound
         d.flo = d.k;
         if (d.ceil <= d.k) d.ceil = 0xffu;  // the clip bound overrides the waste ceiling
+        d.changed = true;
+    } else if (wasteful && k > flo && steps >= 4 * p.settle) {
+        // sustained waste while the head does not move (one bucket holding the whole frontier:
+        // RMAT with U[1,2^20] re-expanded 6x at 2^15 with the head parked for 20 ms): shrink
+        // after four settling periods even without head switches
+        d.k = k - 1;
+        d.ceil = k;
         d.changed = true;
     } else if (steps >= p.settle && turned) {
         if (wasteful && k > flo) {
@@ -218,12 +225,23 @@ __device__ __forceinline__ long long bucket_pending(const Params<DistT>& p, unsi
     return (long long)(r + l - d);
 }
 
+// Re-expansion share of the recent window.  A window too small to measure (a crawling run
+// or a drain) keeps the last measured share: an unmeasurable window must not read as
+// "no waste" once the run has shown waste (ER with degree 4 grew Delta 2^21 -> 2^25 in its
+// drain on such readings, profiles/r02_sweeps.md §7); before any measurement it is unknown.
 template <typename DistT>
 __device__ __forceinline__ unsigned recent_waste(const Params<DistT>& p, bool& known) {
     const unsigned long long e = ld_relaxed_u64(&p.ctl->g_exp) - ld_relaxed_u64(&p.ctl->exp_mark);
     const unsigned long long f = ld_relaxed_u64(&p.ctl->g_first) - ld_relaxed_u64(&p.ctl->first_mark);
-    known = e >= 4096;
-    return (known && e > f) ? (unsigned)((e - f) * 1000ull / e) : 0u;
+    if (e >= 4096) {
+        known = true;
+        const unsigned w = e > f ? (unsigned)((e - f) * 1000ull / e) : 0u;
+        st_relaxed_u32(&p.ctl->last_waste, w + 1u);
+        return w;
+    }
+    const unsigned lw = ld_relaxed_u32(&p.ctl->last_waste);
+    known = lw != 0u;
+    return known ? lw - 1u : 0u;
 }
 template <typename DistT>
 __device__ __forceinline__ unsigned cumulative_ratio(const Params<DistT>& p) {
@@ -314,7 +332,7 @@ __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lan
     const unsigned clip = recent_clip(p, cknown);
     const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), meta_ceil(hd.meta), true, total, tail, win, waste,
                                  known, clip, cknown, cumulative_ratio(p),
-                                 ld_relaxed_u64(&p.ctl->g_first) >= p.startup_first ||
+                                 ld_relaxed_u64(&p.ctl->g_exp) >= p.startup_first ||
                                      ld_relaxed_u32(&p.ctl->head_switches) >= 32u,
                                  (long long)ld_relaxed_u64(&p.ctl->g_busy));
     const Head nhd{rehead(hd.h + o, k, d.k),
@@ -341,7 +359,7 @@ __device__ void periodic_step(const Params<DistT>& p, const int lane) {
     const unsigned clip = recent_clip(p, cknown);
     const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), meta_ceil(hd.meta), false, total, tail, win, waste,
                                  known, clip, cknown, cumulative_ratio(p),
-                                 ld_relaxed_u64(&p.ctl->g_first) >= p.startup_first ||
+                                 ld_relaxed_u64(&p.ctl->g_exp) >= p.startup_first ||
                                      ld_relaxed_u32(&p.ctl->head_switches) >= 32u,
                                  (long long)ld_relaxed_u64(&p.ctl->g_busy));
     const Head nhd{rehead(hd.h, k, d.k), pack_meta(hs, d.k, d.A, d.flo, d.since, d.ceil)};

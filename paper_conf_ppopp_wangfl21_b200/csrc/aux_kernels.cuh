@@ -79,6 +79,7 @@ __global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned s
             ctl->g_exp = ctl->g_first = ctl->exp_mark = ctl->first_mark = 0;
             ctl->g_push = ctl->g_clip = ctl->push_mark = ctl->clip_mark = 0;
             ctl->g_busy = 0;
+            ctl->last_waste = 0;
             ctl->last_ctl_ns = ctl->t_start;
             ctl->st_vertices = ctl->st_edges = ctl->st_pushes = ctl->st_stale = ctl->st_local = 0;
             ctl->reach_v = ctl->reach_e = ctl->max_dist = 0;

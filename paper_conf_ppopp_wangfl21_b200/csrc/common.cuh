@@ -122,7 +122,8 @@ struct alignas(128) Ctl {
     unsigned long long g_clip;    // items pushed into the tail bucket (clipped)
     char pad8_[120];
     unsigned long long g_busy;    // CTAs holding a batch (the paper's "work assigned")
-    char pad9_[120];
+    unsigned last_waste;          // last measured re-expansion share + 1 (0 = never measured)
+    char pad9_[116];
     unsigned long long st_local;  // items continued CTA-locally
     // statistics (flushed once per CTA at exit, or by finalize)
     unsigned long long st_vertices, st_edges, st_pushes, st_stale;

@@ -429,12 +429,13 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     // and 1 on road-like graphs, where 2 gained only 2 % with more run-to-run spread and 3 sent
     // the controller into a shrink spiral
     const unsigned A0 = g->opts.active_init ? g->opts.active_init : (g->m > 8ull * g->n ? 4u : 1u);
-    // initial floor of Delta (the controller never shrinks below it): the ring-span
-    // value w_max / B, below which one maximum-weight hop from the head already
-    // lands beyond the ring and is clipped ("the value of Delta should
-    // be large enough to minimize the chance of clipping"; reading R8)
+    // initial floor of Delta (the controller never shrinks below it; clipping raises it):
+    // 8x below the ring-span value w_max / B (below which one maximum-weight hop from the head
+    // lands beyond the ring).  Graphs whose distances are made of small weights need the
+    // room: RMAT with U[1,2^20] has its best static Delta at or below 2^13 with the span at 2^15
+    // (reading R8, profiles/r02_sweeps.md §7)
     const unsigned span = kF ? heuristic_k(g) : g->heur_k_span;
-    Head h0{0ull, pack_meta(0, k, A0, std::min(k, span), 0)};
+    Head h0{0ull, pack_meta(0, k, A0, std::min(k, span > 3 ? span - 3 : 0u), 0)};
     Params<DistT> p = make_params<DistT>(g, w, grid, bt, k_max, conc);
     p.a_min = A0;
     p.a_max = std::min(g->opts.num_buckets, std::max(2u, 2u * A0));
