@@ -47,7 +47,7 @@ def main():
     rnd = sys.argv[1] if len(sys.argv) > 1 else "r01"
     src = os.path.join(ROOT, "gpurun_out")
     summary, lines = {}, []
-    for cfg in ("road", "rmat", "er"):
+    for cfg in ("road", "rmat", "er", "batch"):
         rep = os.path.join(src, f"{rnd}_full_{cfg}.ncu-rep")
         if not os.path.exists(rep):
             continue
@@ -58,7 +58,9 @@ def main():
         rd = get("dram__bytes_read.sum") * scale.get(unit("dram__bytes_read.sum"), 1)
         wr = get("dram__bytes_write.sum") * scale.get(unit("dram__bytes_write.sum"), 1)
         st = stalls(rep)
-        summary[cfg] = {"dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
+        shape = lambda k: int(float(m[k][0])) if k in m else None  # noqa: E731
+        summary[cfg] = {"block": shape("launch__block_size"), "grid": shape("launch__grid_size"), "round": rnd,
+                        "dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
                         "duration_ms_under_ncu": get("gpu__time_duration.sum"),
                         "metrics": {k: m[k][0] + " " + m[k][1] for k in WANT if k in m}, "stalls_pct": st}
         lines.append(f"== {cfg}: persistent kernel, one launch, ncu --set full ({rnd})")
@@ -68,7 +70,7 @@ def main():
         lines.append(f"  dram read+write per launch: {(rd + wr) / 1e9:.3f} GB")
         lines.append("  top stall reasons (% of samples): " + ", ".join(f"{k}={v}" for k, v in st.items()))
     # launch list: share of the persistent kernel in the step
-    lc = os.path.join(src, f"{rnd}_launches_road.csv")
+    lc = os.path.join(src, f"{rnd}_launches.csv")
     if os.path.exists(lc):
         rows = [r for r in csv.reader(open(lc)) if len(r) > 10]
         h = rows[0]
@@ -78,12 +80,12 @@ def main():
             name = r[ik].split("(")[0].split("<")[0].replace("void ", "").strip()
             per.setdefault(name, []).append(float(r[iv].replace(",", "")))
         tot = sum(sum(v) for v in per.values())
-        lines.append(f"== launch list of `bench.py --steps 2 --warmup 1` (road), ncu gpu__time_duration ({rnd})")
+        lines.append(f"== launch list of `bench.py --steps 1 --warmup 3` (default workload), ncu gpu__time_duration ({rnd})")
         share = {}
         for k, v in sorted(per.items(), key=lambda x: -sum(x[1])):
             share[k] = {"launches": len(v), "total_ns": sum(v), "share": sum(v) / tot}
             lines.append(f"  {k:45s} launches={len(v):3d} total={sum(v) / 1e6:9.3f} ms share={100 * sum(v) / tot:5.1f}%")
-        summary["launch_list_road"] = share
+        summary["launch_list"] = share
     os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
     with open(os.path.join(ROOT, "profiles", f"{rnd}_ncu_summary.txt"), "w") as f:
         f.write("\n".join(lines) + "\n")
