@@ -631,8 +631,12 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     __shared__ unsigned s_cnt[kMaxBuckets];
     __shared__ unsigned long long s_base[kMaxBuckets];
     __shared__ unsigned s_wsum[kWarps], s_wnz[kWarps];
-    __shared__ unsigned s_total, s_E, s_NZ, s_got, s_slot, s_lnext, s_direct, s_task, s_ahead;
-    __shared__ int s_cmd;
+    __shared__ unsigned s_total, s_E, s_NZ, s_got, s_slot, s_lnext, s_direct, s_task, s_tslot;
+    __shared__ volatile unsigned s_ahead;  // (own load: not merged with the claim fields)
+    __shared__ int s_cmd[2];  // by loop parity: an idle CTA loops back to the claim with no
+                              // second barrier, so the next claim must not overwrite the
+                              // value a slow warp is still to read (compute-sanitizer racecheck)
+    unsigned par = 0;
     __shared__ unsigned long long s_idx;
     __shared__ Head s_head;
     __shared__ unsigned long long s_prof[kProfCounters];
@@ -716,10 +720,11 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                         __nanosleep(backoff);
                     }
                 }
-                if (lane == 0) s_cmd = cmd;
+                if (lane == 0) s_cmd[par] = cmd;
             }
             __syncthreads();
-            const int cmd = s_cmd;
+            const int cmd = s_cmd[par];
+            par ^= 1u;
             if (prof) {
                 const long long t1 = clock64();
                 s_prof[cmd == CMD_WORK ? PR_CLAIM : PR_IDLE] += t1 - t0;
@@ -754,12 +759,12 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             // a hub-split chunk: one vertex, len arcs, charged to the slot it carries
             if (tid == 0) {
                 SplitTask* tp = p.tasks + (s_idx & (p.tcap - 1));
-                s_slot = 0;
+                s_tslot = 0;  // (not s_slot: other threads may still be reading it)
                 const unsigned len = take_chunk(p, tp);
                 if (len) {
                     const unsigned long long b = __ldcg(&tp->beg), d = __ldcg(&tp->d);
                     const unsigned v = __ldcg(&tp->v);
-                    s_slot = __ldcg(&tp->slot);
+                    s_tslot = __ldcg(&tp->slot);
                     st_release_u32(&tp->len, 0u);  // free the slot after the read
                     const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
                     if (cur >= d) {  // stale chunks (v improved since) are dropped
@@ -862,7 +867,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             s_d[r] = (DistT)my_d;
         }
         const unsigned E = s_E, NZ = s_NZ;
-        if (is_task) slot = s_slot;
+        if (is_task) slot = s_tslot;
         const int nexp = is_task ? 0 : nlive;  // a chunk is not a vertex expansion
         if (tid == 0) {
             c_vert += nexp;
@@ -989,6 +994,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             // bucket (s_wcnt[warp]): deferred from the push sites to here, where a warp-wide
             // match_any covers 32 staged items instead of the one or two pushes of a site.
             auto rank_segment = [&]() {
+                __syncwarp();  // staged entries written by other lanes (emit) are visible
                 for (unsigned i0 = 0; i0 < wfill; i0 += 32) {
                     const unsigned i = i0 + (unsigned)lane;
                     const unsigned my = (unsigned)warp * kSeg + i;
@@ -1190,6 +1196,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             // Rows longer than kWDeg go back through the ring (head bucket).
             constexpr unsigned kWDeg = 8u * EPT;
             if constexpr (WLC) while (wq_n > 0) {
+                __syncwarp();  // the queue entries written by other lanes (keep) are visible
                 const unsigned take = wq_n < 32u ? wq_n : 32u;
                 const unsigned st0 = wq_h;  // logical start of this hop's items
                 const unsigned ph = wq0 + (st0 + lane) % kWQ;
@@ -1363,11 +1370,11 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     tq += clock64() - tf;
                     s_prof[PR_N_FLUSH] += 1;
                 }
-            } else if (p.dynamic && tid == 0 && s_direct) {
-                atomicAdd(&p.ctl->g_push, (unsigned long long)s_direct);
             }
-            if (tid == 0) {
-                c_push += total + s_direct;
+            if (tid == 0) {  // (s_direct is read by thread 0 only: it also resets it)
+                const unsigned direct = s_direct;
+                if (!any_staged && p.dynamic && direct) atomicAdd(&p.ctl->g_push, (unsigned long long)direct);
+                c_push += total + direct;
                 s_total = 0;
                 s_direct = 0;
             }
@@ -1385,8 +1392,12 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         // s_lnext final (also covers the E == 0 case); first expansions for the controller
         const int nfirst = __syncthreads_count(fbit != 0 && (fword & fbit) == 0);
         const unsigned kept = s_lnext < lcap ? s_lnext : lcap;
-        const unsigned w_exp = s_wst[0], w_first = s_wst[1], w_kept = s_wst[4];
+        // (thread 0 alone reads the warp-local counters: it also resets them below)
+        unsigned w_exp = 0, w_first = 0, w_kept = 0;
         if (tid == 0) {
+            w_exp = s_wst[0];
+            w_first = s_wst[1];
+            w_kept = s_wst[4];
             if (wlc) {
                 c_vert += w_exp;
                 c_edges += s_wst[2];
