@@ -382,6 +382,32 @@ __device__ __forceinline__ unsigned long long relax_sum(unsigned long long d, un
 }
 // a sum that can never be an improvement (float: +inf / NaN) or that overflows
 // the distance type (integer: re-run with 64-bit distances)
+// The same sum in the distance type's width.  bad = the sum is no distance this run can store:
+// float +inf/NaN (never an improvement) or an integer sum that reaches the 32-bit infinity
+// value or wraps (the host re-runs with 64-bit distances).  64-bit sums cannot wrap: a distance
+// is at most (n-1)(2^32-1) < 2^64 - 2^32.
+template <bool kF, typename DistT>
+__device__ __forceinline__ DistT relax_narrow(DistT d, unsigned w, bool& bad) {
+    if constexpr (kF) {
+        const unsigned s = __float_as_uint(__fadd_rn(__uint_as_float((unsigned)d), __uint_as_float(w)));
+        bad = s >= 0x7F800000u;
+        return (DistT)s;
+    } else if constexpr (sizeof(DistT) == 4) {
+        const unsigned s = (unsigned)d + w;
+        bad = s < w || s == 0xFFFFFFFFu;
+        return s;
+    } else {
+        const unsigned long long s = (unsigned long long)d + w;
+        bad = s == ~0ull;
+        return s;
+    }
+}
+template <typename DistT>
+struct alignas(16) ItemInfo {
+    unsigned long long eadj;  // row begin - the item's first arc index in the batch
+    DistT d;                  // the item's distance
+};
+
 template <bool kF>
 __device__ __forceinline__ bool sum_unusable(unsigned long long nd, unsigned long long inf) {
     if constexpr (kF) return nd >= 0x7F800000ull;
@@ -566,9 +592,8 @@ struct Smem {
     static constexpr size_t o_arc = 0;                                        // (no arc window)
     static constexpr size_t o_items = 0;                                      // Raw[kStage] staged pushes
     // per expanded item (compacted: items with at least one arc, in scan order)
-    static constexpr size_t o_ebeg = o_items + align16((size_t)kStage * sizeof(Raw));  // u64[BT] row begin - scan
-    static constexpr size_t o_d = o_ebeg + (size_t)BT * 8;                    // DistT[BT] item distance
-    static constexpr size_t o_ld = o_d + align16((size_t)BT * sizeof(DistT));  // DistT[BT] kept children
+    static constexpr size_t o_info = o_items + align16((size_t)kStage * sizeof(Raw));  // ItemInfo[BT]
+    static constexpr size_t o_ld = o_info + (size_t)BT * 16;                  // DistT[BT] kept children
     static constexpr size_t o_owner = o_ld + align16((size_t)BT * sizeof(DistT));  // (unused)
     static constexpr size_t o_rank = o_owner;                                 // u16[kStage]
     static constexpr size_t o_scan = o_rank + align16((size_t)kStage * 2);    // u32[BT+1] arc offsets, sentinel E
@@ -608,8 +633,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
 
     extern __shared__ __align__(16) unsigned char smem[];
     Raw* s_items = (Raw*)(smem + L::o_items);
-    unsigned long long* s_eadj = (unsigned long long*)(smem + L::o_ebeg);  // row begin - arc offset
-    DistT* s_d = (DistT*)(smem + L::o_d);
+    // per expanded item, one 16-byte shared load per arc: {row begin - arc offset, distance}
+    ItemInfo<DistT>* s_info = (ItemInfo<DistT>*)(smem + L::o_info);
     DistT* s_ld = (DistT*)(smem + L::o_ld);
     unsigned short* s_rank = (unsigned short*)(smem + L::o_rank);
     unsigned* s_scan = (unsigned*)(smem + L::o_scan);
@@ -863,8 +888,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             const unsigned r = s_wnz[warp] + __popc(nzm & lt_mask);
             const unsigned ex = x - deg + s_wsum[warp];
             s_scan[r] = ex;
-            s_eadj[r] = my_b - ex;  // arc e of the batch is adj[s_eadj[owner] + e]
-            s_d[r] = (DistT)my_d;
+            s_info[r] = ItemInfo<DistT>{my_b - ex, (DistT)my_d};  // arc e of the batch is adj[eadj + e]
         }
         const unsigned E = s_E, NZ = s_NZ;
         if (is_task) slot = s_tslot;
@@ -882,7 +906,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             tw = 0;
         }
 
-        __syncthreads();  // publishes s_scan / s_d / s_eadj
+        __syncthreads();  // publishes s_scan / s_info
         if (CA && tid == 0) s_ahead = 0;  // every thread has read it (loop top)
         unsigned wfill = 0;  // warp-uniform: items staged in this warp's segment
         // ---------------------------------------------------- stream the batch's arcs
@@ -917,7 +941,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
                 cur = lo;
             }
-            auto fetch = [&](unsigned base, unsigned (&own)[EPT], uint2 (&a)[EPT]) {
+            auto fetch = [&](unsigned base, DistT (&dv)[EPT], uint2 (&a)[EPT]) {
+                unsigned own[EPT];
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {
                     const unsigned w0 = base + j * 32;
@@ -930,7 +955,13 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {  // EPT independent arc loads in flight
                     const unsigned e = base + j * 32 + lane;
-                    a[j] = e < we ? ld_stream_u2(p.adj + (s_eadj[own[j]] + e), pol_stream) : make_uint2(0u, 0u);
+                    a[j] = make_uint2(0u, 0u);
+                    dv[j] = (DistT)0;
+                    if (e < we) {
+                        const ItemInfo<DistT> ii = s_info[own[j]];
+                        a[j] = ld_stream_u2(p.adj + (ii.eadj + e), pol_stream);
+                        dv[j] = ii.d;
+                    }
                 }
             };
             // head-bucket children stay on chip: first in this warp's own queue (warp-local
@@ -1096,27 +1127,32 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             // result).  Without the gather (tiny batches) or with the 16-bit filter (cur is
             // only a bound) the returning atomicMin decides.
             const bool fire = !tiny && p.filt == nullptr;
-            auto body = [&](const unsigned base, const unsigned (&own)[EPT], const uint2 (&a)[EPT]) {
-                unsigned long long nd[EPT];
+            // (distances in DistT width: d + w is computed in 32 bits for 32-bit distances, an
+            // overflow or the infinity value flags a re-run with 64-bit distances)
+            auto body = [&](const unsigned base, const DistT (&dv)[EPT], const uint2 (&a)[EPT]) {
+                DistT nd[EPT];
+                bool live[EPT], bad[EPT];
                 bool push[EPT];
                 DistT cur[EPT];
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {
-                    const unsigned e = base + j * 32 + lane;
-                    nd[j] = e < we ? relax_sum<kF>((unsigned long long)s_d[own[j]], a[j].y) : kInf;
+                    live[j] = base + j * 32 + lane < we;
+                    nd[j] = relax_narrow<kF, DistT>(dv[j], a[j].y, bad[j]);
+                    bad[j] = bad[j] && live[j];
+                    live[j] = live[j] && !bad[j];
                 }
 #pragma unroll
                 for (int j = 0; j < EPT; ++j)  // EPT independent L2 gathers in flight
-                    cur[j] = nd[j] < kInf ? DistInf<DistT>::value : (DistT)0;
+                    cur[j] = live[j] ? DistInf<DistT>::value : (DistT)0;
                 if (!tiny) {
                     if (p.filt == nullptr) {  // (uniform branch: the opt-in filter path stays out of the loop)
 #pragma unroll
                         for (int j = 0; j < EPT; ++j)
-                            if (nd[j] < kInf) cur[j] = ld_keep(p.dist + a[j].x, pol_keep);
+                            if (live[j]) cur[j] = ld_keep(p.dist + a[j].x, pol_keep);
                     } else {
 #pragma unroll
                         for (int j = 0; j < EPT; ++j)
-                            if (nd[j] < kInf)
+                            if (live[j])
                                 cur[j] = (DistT)min(filt_bound(ld_filt(p.filt + a[j].x), p.filt_shift),
                                                     (unsigned long long)DistInf<DistT>::value);
                     }
@@ -1125,20 +1161,19 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 bool tried[EPT];
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {  // all atomics issued before any result is used
-                    const unsigned e = base + j * 32 + lane;
                     tried[j] = false;
                     old[j] = (DistT)0;
-                    if (e < we) {
-                        if (sum_unusable<kF>(nd[j], kInf)) {
-                            if (!kF) atomicOr(&p.ctl->status, kStDistOverflow);  // 32-bit distances insufficient
-                        } else if (nd[j] < (unsigned long long)cur[j]) {
+                    if (bad[j]) {
+                        if (!kF) atomicOr(&p.ctl->status, kStDistOverflow);  // 32-bit distances insufficient
+                    } else if (live[j]) {
+                        if (nd[j] < cur[j]) {
                             if (fire) {
-                                // fire-and-forget (D17): push on the gathered value; the RED
+                                // fire-and-forget (D19): push on the gathered value; the RED
                                 // needs no round trip
-                                red_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
+                                red_min_keep(p.dist + a[j].x, nd[j], pol_keep);
                                 old[j] = cur[j];
                             } else {
-                                old[j] = atomic_min_keep(p.dist + a[j].x, (DistT)nd[j], pol_keep);
+                                old[j] = atomic_min_keep(p.dist + a[j].x, nd[j], pol_keep);
                             }
                             tried[j] = true;
                         }
@@ -1146,42 +1181,42 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {
-                    push[j] = tried[j] && nd[j] < (unsigned long long)old[j];
+                    push[j] = tried[j] && nd[j] < old[j];
                     if (push[j] && p.filt) st_filt(p.filt + a[j].x, filt_enc(nd[j], p.filt_shift));
                 }
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {
                     if (!__any_sync(FULL, push[j])) continue;
-                    const unsigned o = push[j] ? bucket_of<kF>(nd[j], k, hd.h, p.nb) : 0u;
-                    const bool kept = keep(push[j] && o == 0, a[j].x, nd[j], false, 0ull, 0u);
-                    emit(push[j] && !kept, a[j].x, nd[j], o);
+                    const unsigned o = push[j] ? bucket_of<kF>((unsigned long long)nd[j], k, hd.h, p.nb) : 0u;
+                    const bool kept = keep(push[j] && o == 0, a[j].x, (unsigned long long)nd[j], false, 0ull, 0u);
+                    emit(push[j] && !kept, a[j].x, (unsigned long long)nd[j], o);
                 }
             };
             if (PIPE && we > wb + kChunk) {
                 // software pipeline: round r+1's owners and arc loads are issued before
                 // round r's gathers and atomics
-                unsigned own_n[EPT];
+                DistT dv_n[EPT];
                 uint2 a_n[EPT];
-                if (wb < we) fetch(wb, own_n, a_n);
+                if (wb < we) fetch(wb, dv_n, a_n);
                 for (unsigned base = wb; base < we;) {
-                    unsigned own[EPT];
+                    DistT dv[EPT];
                     uint2 a[EPT];
 #pragma unroll
                     for (int j = 0; j < EPT; ++j) {
-                        own[j] = own_n[j];
+                        dv[j] = dv_n[j];
                         a[j] = a_n[j];
                     }
                     const unsigned nxt = base + kChunk;
-                    if (nxt < we) fetch(nxt, own_n, a_n);
-                    body(base, own, a);
+                    if (nxt < we) fetch(nxt, dv_n, a_n);
+                    body(base, dv, a);
                     base = nxt;
                 }
             } else {
                 for (unsigned base = wb; base < we; base += kChunk) {
-                    unsigned own[EPT];
+                    DistT dv[EPT];
                     uint2 a[EPT];
-                    fetch(base, own, a);
-                    body(base, own, a);
+                    fetch(base, dv, a);
+                    body(base, dv, a);
                 }
             }
             // ------------------------------------------------ warp-local continuation
