@@ -85,6 +85,10 @@ typedef enum sssp_status {
                                         controller varies the number of active buckets between
                                         the degree-based default A0 and 2*A0 from the CTAs holding work */
 #define SSSP_FLAG_FIXED_ACTIVE 0x1000u /* ablation: keep the active-bucket count at its initial value */
+#define SSSP_FLAG_CHUNKED_RING 0x2000u /* bucket storage as a shared pool of 4096-item chunks (the paper's
+                                        block pool): memory bounded by the items alive at
+                                        once (default pool 2n items, grown x2 on exhaustion) instead of
+                                        one no-lap array of >= n items per bucket (32n items) */
 #define SSSP_FLAG_L2_PERSIST 0x20u /* reserve the L2 persisting set-aside for dist (raises the device-wide
                                      cudaLimitPersistingL2CacheSize to min(dist bytes, maximum)) and mark
                                      dist accesses evict_last.  Off by default: measured on B200
@@ -136,7 +140,9 @@ typedef struct sssp_options {
     uint32_t dist_bits;        /* 0 = auto (32-bit internal distances when provably or observably
                                   safe, else 64), 32 or 64 */
     uint64_t ring_items;       /* capacity of each bucket's circular array (items, rounded up to a
-                                  power of two, >= 64); 0 = auto = max(2^16, next_pow2(n)) */
+                                  power of two, >= 64); 0 = auto = max(2^16, next_pow2(n)).  With
+                                  SSSP_FLAG_CHUNKED_RING: items of the shared chunk pool (>= 64
+                                  chunks of 4096); 0 = auto = max(2^18, next_pow2(2n)) */
     uint32_t flags;            /* SSSP_FLAG_* */
     uint32_t block_threads;    /* worker CTA size: 0 = auto (512; 128 on road-like graphs), else 128/256/512/1024 */
     uint32_t grid_ctas;        /* 0 = every co-resident CTA; else at most this many CTAs */
@@ -195,6 +201,8 @@ typedef struct sssp_stats {
     float batch_ms;              /* device time of the whole call on the caller's stream (CUDA events) */
     uint32_t concurrency;        /* sources that were in flight at once */
     uint32_t worker;             /* SSSP_WORKER_CTA: the worker granularity that ran */
+    uint64_t ring_bytes;         /* device bytes of one workspace's bucket storage (items + chunk
+                                    tables); the run used max(1, concurrency) workspaces */
 } sssp_stats;
 
 /* One Delta-controller sample (written at each head-bucket switch and at each

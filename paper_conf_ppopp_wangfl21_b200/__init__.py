@@ -35,6 +35,7 @@ SSSP_FLAG_PROFILE = 0x10
 SSSP_FLAG_L2_PERSIST = 0x20
 SSSP_FLAG_ADAPT_ACTIVE = 0x40  # (default since round 2)
 SSSP_FLAG_FIXED_ACTIVE = 0x1000
+SSSP_FLAG_CHUNKED_RING = 0x2000
 SSSP_FLAG_NO_WARP_LOCAL = 0x80
 SSSP_FLAG_WARP_LOCAL = 0x100
 SSSP_FLAG_FILTER16 = 0x200
@@ -93,7 +94,7 @@ class sssp_stats(ctypes.Structure):
         ("dist_bits", ctypes.c_uint32), ("grid_ctas", ctypes.c_uint32), ("block_threads", ctypes.c_uint32),
         ("runs", ctypes.c_uint32), ("trace_entries", ctypes.c_uint32), ("kernel_ms", ctypes.c_float),
         ("total_ms", ctypes.c_float), ("status", ctypes.c_uint32), ("batch_ms", ctypes.c_float),
-        ("concurrency", ctypes.c_uint32), ("worker", ctypes.c_uint32),
+        ("concurrency", ctypes.c_uint32), ("worker", ctypes.c_uint32), ("ring_bytes", ctypes.c_uint64),
     ]
 
 

@@ -84,6 +84,14 @@ struct Params {
     SplitTask* tasks;          // hub-split chunk queue (counters in bk[kSplitQ])
     unsigned long long tcap;   // entries, power of two
     unsigned split_deg;        // split vertices with more arcs than this (0 = off)
+    // chunked bucket storage (0 = one no-lap array of cap items per bucket, D13)
+    unsigned chunked;
+    unsigned* ctab;            // nb x (tab_mask + 1): chunk id + 1 (0 = not taken yet)
+    unsigned tab_mask;
+    unsigned* chunk_used;      // items read per chunk
+    unsigned* free_ring;       // pool_chunks entries: chunk id + 1 (0 = empty)
+    ChunkPool* pool;
+    unsigned pool_chunks;      // power of two
     unsigned k_max;
     unsigned long long timeout_ns;
 };
@@ -172,7 +180,7 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
         d.flo = d.k;
         if (d.ceil <= d.k) d.ceil = 0xffu;  // the clip bound overrides the waste ceiling
         d.changed = true;
-    } else if (wasteful && k > flo && steps >= 4 * p.settle) {
+    } else if (wasteful && k > flo && steps >= 4 * p.settle && hsw == 0) {
         // sustained waste while the head does not move (one bucket holding the whole frontier:
         // RMAT with U[1,2^20] re-expanded 6x at 2^15 with the head parked for 20 ms): shrink
         // after four settling periods even without head switches
@@ -526,6 +534,97 @@ __device__ unsigned claim_batch(const Params<DistT>& p, int lane, unsigned& o_sl
     return 0;
 }
 
+// --------------------------------------------------------------- bucket storage
+// Where item idx of ring slot sl lives.  Flat (default): slot sl's own array of cap items,
+// never lapped within a run (D13).  Chunked: through the slot's chunk table; the chunk is
+// published by its reserver before any of its items is stored or claimed, so a wait here is
+// only for that publication to become visible.  nullptr = the run was aborted while waiting.
+template <typename DistT>
+__device__ __forceinline__ char* item_ptr(const Params<DistT>& p, unsigned sl, unsigned long long idx, bool chk) {
+    constexpr int kB = ItemT<DistT>::kBytes;
+    if (!chk) return p.ring + ((size_t)sl * p.cap + (idx & (p.cap - 1))) * kB;
+    const unsigned* e = p.ctab + (size_t)sl * (p.tab_mask + 1) + ((idx >> kChunkShift) & p.tab_mask);
+    unsigned id1, spins = 0;
+    while ((id1 = ld_acquire_u32(e)) == 0u)
+        if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) return nullptr;
+    return p.ring + (((size_t)(id1 - 1) << kChunkShift) + (idx & (kChunkItems - 1))) * kB;
+}
+// A reserve of [b, b + c) overflows the flat array (no laps, D13); chunked storage overflows
+// only when the pool is exhausted (chunk_alloc).
+template <typename DistT>
+__device__ __forceinline__ bool flat_overflow(const Params<DistT>& p, unsigned long long b, unsigned long long c, bool chk) {
+    return !chk && b + c > p.cap;
+}
+template <typename DistT>
+__device__ unsigned chunk_alloc(const Params<DistT>& p) {
+    const unsigned long long f = atomicAdd(&p.pool->fresh.v, 1ull);
+    if (f < p.pool_chunks) return (unsigned)f;
+    const long long old = (long long)atomicAdd(&p.pool->favail.v, (unsigned long long)(-1ll));
+    if (old <= 0) {
+        atomicAdd(&p.pool->favail.v, 1ull);
+        atomicOr(&p.ctl->status, kStRingOverflow);  // pool exhausted: the host doubles it and re-runs
+        return 0xFFFFFFFFu;
+    }
+    const unsigned long long c = atomicAdd(&p.pool->fclaim.v, 1ull);
+    unsigned* e = p.free_ring + (c & (p.pool_chunks - 1));
+    unsigned id1, spins = 0;
+    while ((id1 = ld_acquire_u32(e)) == 0u)
+        if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) return 0xFFFFFFFFu;
+    st_relaxed_u32(e, 0u);
+    return id1 - 1;
+}
+// After a reserve of [b, b + c) in slot sl: take every chunk whose first index is in the range
+// (the range that reserved a chunk's first index is its only taker).
+template <typename DistT>
+__device__ void chunks_for_range(const Params<DistT>& p, unsigned sl, unsigned long long b, unsigned long long c,
+                                 bool chk) {
+    if (!chk || c == 0) return;
+    for (unsigned long long ci = (b + kChunkItems - 1) >> kChunkShift; (ci << kChunkShift) < b + c; ++ci) {
+        const unsigned id = chunk_alloc(p);
+        if (id == 0xFFFFFFFFu) return;
+        unsigned* e = p.ctab + (size_t)sl * (p.tab_mask + 1) + (ci & p.tab_mask);
+        // the table entry of chunk ci - T must be free by now (T >= pool chunks); if a lagging
+        // reader still held it, abort the run rather than alias two chunks
+        if (atomicCAS(e, 0u, id + 1) != 0u) atomicOr(&p.ctl->status, kStRingOverflow);
+    }
+}
+// Chunk id (+1) of item idx of slot sl, waiting for its publication (0 = aborted run).
+template <typename DistT>
+__device__ __forceinline__ unsigned chunk_of(const Params<DistT>& p, unsigned sl, unsigned long long idx) {
+    const unsigned* e = p.ctab + (size_t)sl * (p.tab_mask + 1) + ((idx >> kChunkShift) & p.tab_mask);
+    unsigned id1, spins = 0;
+    while ((id1 = ld_acquire_u32(e)) == 0u)
+        if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) return 0u;
+    return id1;
+}
+template <typename DistT>
+__device__ __forceinline__ char* chunk_item(const Params<DistT>& p, unsigned id1, unsigned long long idx) {
+    return p.ring + (((size_t)(id1 - 1) << kChunkShift) + (idx & (kChunkItems - 1))) * ItemT<DistT>::kBytes;
+}
+
+// Thread 0, after the CTA barrier that follows a pop of [idx0, idx0 + got) in slot sl (every
+// item read and cleared): count the reads per chunk; the reader that completes a chunk frees it.
+template <typename DistT>
+__device__ void chunks_consumed(const Params<DistT>& p, unsigned sl, unsigned long long idx0, unsigned got) {
+    const unsigned long long end = idx0 + got;
+    for (unsigned long long i = idx0; i < end;) {
+        const unsigned long long cend = ((i >> kChunkShift) + 1) << kChunkShift;
+        const unsigned cnt = (unsigned)((cend < end ? cend : end) - i);
+        unsigned* e = p.ctab + (size_t)sl * (p.tab_mask + 1) + ((i >> kChunkShift) & p.tab_mask);
+        const unsigned id1 = ld_relaxed_u32(e);  // still ours: not all of its items are counted yet
+        __threadfence();                         // the CTA's clears (barrier-ordered) before the count
+        if (atomicAdd(p.chunk_used + (id1 - 1), cnt) + cnt == kChunkItems) {
+            p.chunk_used[id1 - 1] = 0;
+            st_relaxed_u32(e, 0u);
+            __threadfence();
+            const unsigned long long r = atomicAdd(&p.pool->freserve.v, 1ull);
+            st_release_u32(p.free_ring + (r & (p.pool_chunks - 1)), id1);
+            atomicAdd(&p.pool->favail.v, 1ull);
+        }
+        i += cnt;
+    }
+}
+
 // --------------------------------------------------------------- hub split (A5)
 // Publish arcs [S, deg) of vertex v (expanded at distance d, row begins at b) as
 // chunks of S arcs; the caller processes the first S itself.  The chunks are
@@ -620,7 +719,9 @@ struct Smem {
 // has streamed its own slice of the current one, so the claim round trips overlap the
 // other warps' streaming, the flush and the completion (held for the tail of one batch
 // only; claiming at the start of a batch held the claim too long, sweeps §7).
-template <typename DistT, int BT, int EPT, int MINB, bool PIPE, bool kF, bool WLC = true, bool CA = false>
+// CHM: bucket storage -- 0 flat no-lap arrays, 1 chunked pool, 2 chosen at run time (p.chunked);
+// the product's default builds are compiled for 0 and 1 so the flat path carries no chunk code.
+template <typename DistT, int BT, int EPT, int MINB, bool PIPE, bool kF, bool WLC = true, bool CA = false, int CHM = 2>
 __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<DistT> p) {
     // items per thread: one (batches of two items per thread, to pay the per-batch round
     // trips half as often, measured slower -- ER 13.1 vs 11.4 ms -- from register spills)
@@ -655,6 +756,9 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     __shared__ unsigned s_wcnt[kWarps][kMaxBuckets];
     __shared__ unsigned s_cnt[kMaxBuckets];
     __shared__ unsigned long long s_base[kMaxBuckets];
+    // chunks one CTA reservation (<= kStage items) can span
+    constexpr unsigned kFlushChunks = ((unsigned)kStage + kChunkItems - 1) / kChunkItems + 1;
+    __shared__ unsigned s_cid[kMaxBuckets][kFlushChunks];                  // chunked storage: their ids
     __shared__ unsigned s_wsum[kWarps], s_wnz[kWarps];
     __shared__ unsigned s_total, s_E, s_NZ, s_got, s_slot, s_lnext, s_direct, s_task, s_tslot;
     __shared__ volatile unsigned s_ahead;  // (own load: not merged with the claim fields)
@@ -669,6 +773,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const unsigned lt_mask = lanemask_lt();
     const unsigned le_mask = lt_mask | (1u << lane);
+    const bool chk = CHM == 2 ? p.chunked != 0 : CHM == 1;  // chunked bucket storage
     const unsigned nbm = p.nb - 1;
     const unsigned local_max = p.local_max < (unsigned)BT ? p.local_max : (unsigned)BT;
     unsigned long long c_vert = 0, c_edges = 0, c_push = 0, c_stale = 0, c_local = 0;  // thread 0
@@ -806,11 +911,11 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 unsigned long long d;
                 bool loaded = true;
                 if (from_ring) {
-                    const unsigned long long idx = (s_idx + tid) & (p.cap - 1);
-                    char* sp = p.ring + ((size_t)slot * p.cap + idx) * IT::kBytes;
+                    char* sp = item_ptr(p, slot, s_idx + tid, chk);
                     unsigned spins = 0;
                     SSSP_FUZZ_AT(FZ_POP);
-                    while (!(loaded = IT::load(sp, v, d))) {  // reserved, store not landed yet
+                    loaded = false;
+                    while (sp && !(loaded = IT::load(sp, v, d))) {  // reserved, store not landed yet
                         if ((++spins & 1023) == 0 && ld_relaxed_u32(&p.ctl->status)) break;  // aborted run
                     }
                     if (loaded) IT::clear(sp);  // the slot's one reader this run (D13)
@@ -860,6 +965,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             s_wnz[warp] = __popc(nzm);
         }
         const int nlive = __syncthreads_count(live);
+        // chunked storage: this batch's reads (and clears) are complete; count them per chunk
+        if (chk && tid == 0 && from_ring && !is_task) chunks_consumed(p, slot, s_idx, got);
         if (warp == 0) {
             const unsigned ws = lane < kWarps ? s_wsum[lane] : 0;
             const unsigned wn = lane < kWarps ? s_wnz[lane] : 0;
@@ -1051,19 +1158,32 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 if (c) {
                     b = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
                     SSSP_FUZZ_AT(FZ_RESERVE);
-                    if (b + c > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
+                    if (flat_overflow(p, b, c, chk)) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
+                    chunks_for_range(p, sl, b, c, chk);
                     if (p.dynamic && lane == (int)nbm) atomicAdd(&p.ctl->g_clip, (unsigned long long)c);
+                }
+                // chunked storage: a segment's range spans at most two chunks (kSeg <= kChunkItems)
+                unsigned cid0 = 0, cid1 = 0;
+                if (chk && c) {
+                    cid0 = chunk_of(p, sl, b);
+                    if (((b + c - 1) >> kChunkShift) != (b >> kChunkShift)) cid1 = chunk_of(p, sl, b + c - 1);
                 }
                 for (unsigned i0 = 0; i0 < wfill; i0 += 32) {
                     const unsigned i = i0 + (unsigned)lane;
                     const unsigned my = (unsigned)warp * kSeg + i;
                     const unsigned o = i < wfill ? s_soff[my] : 0u;
                     const unsigned long long bo = __shfl_sync(FULL, b, (int)o);
+                    const unsigned c0 = __shfl_sync(FULL, cid0, (int)o), c1 = __shfl_sync(FULL, cid1, (int)o);
                     if (i < wfill) {
                         const unsigned long long idx = bo + s_rank[my];
                         SSSP_FUZZ_AT(FZ_PUBLISH);
                         // the slot's one writer this run (D13); beyond cap the run is aborted
-                        if (idx < p.cap) IT::store(p.ring + ((size_t)((hs + o) & nbm) * p.cap + idx) * IT::kBytes, s_items[my]);
+                        if (chk) {
+                            const unsigned id1 = ((idx >> kChunkShift) == (bo >> kChunkShift)) ? c0 : c1;
+                            if (id1) IT::store(chunk_item(p, id1, idx), s_items[my]);
+                        } else if (idx < p.cap) {
+                            IT::store(item_ptr(p, (hs + o) & nbm, idx, chk), s_items[my]);
+                        }
                     }
                 }
                 __syncwarp();
@@ -1093,14 +1213,18 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                             if (lane == pl) {
                                 const unsigned c = (unsigned)__popc(peers);
                                 b0 = atomicAdd(&p.bk[sl].reserve.v, (unsigned long long)c);
-                                if (b0 + c > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
+                                if (flat_overflow(p, b0, c, chk)) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
+                                chunks_for_range(p, sl, b0, c, chk);
                                 atomicAdd(&s_direct, c);
                                 SSSP_FUZZ_AT(FZ_RESERVE);
                             }
                             b0 = __shfl_sync(peers, b0, pl);
                             const unsigned long long idx = b0 + __popc(peers & lt_mask);
                             // the slot's one writer this run (D13); beyond cap the run is aborted
-                            if (idx < p.cap) IT::store(p.ring + ((size_t)sl * p.cap + idx) * IT::kBytes, IT::make(v, ndv));
+                            if (chk || idx < p.cap) {
+                                char* ip = item_ptr(p, sl, idx, chk);
+                                if (ip) IT::store(ip, IT::make(v, ndv));
+                            }
                             SSSP_FUZZ_AT(FZ_PUBLISH);
                             __syncwarp(peers);
                             if (lane == pl) atomicAdd(&p.bk[sl].avail.v, (unsigned long long)__popc(peers));
@@ -1373,7 +1497,14 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                             const unsigned long long b = atomicAdd(&p.bk[(hs + o) & nbm].reserve.v, (unsigned long long)x);
                             SSSP_FUZZ_AT(FZ_RESERVE);
                             s_base[o] = b;
-                            if (b + x > p.cap) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
+                            if (flat_overflow(p, b, x, chk)) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
+                            chunks_for_range(p, (hs + o) & nbm, b, x, chk);
+                            if (chk) {  // the range's chunks, once, for every store below
+                                for (unsigned q = 0; q < kFlushChunks; ++q) {
+                                    const unsigned long long ci = (b >> kChunkShift) + q;
+                                    s_cid[o][q] = (ci << kChunkShift) < b + x ? chunk_of(p, (hs + o) & nbm, ci << kChunkShift) : 0u;
+                                }
+                            }
                             if (p.dynamic && o == nbm) atomicAdd(&p.ctl->g_clip, (unsigned long long)x);
                         }
                     }
@@ -1388,7 +1519,12 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     const unsigned long long idx = s_base[o] + s_wcnt[warp][o] + s_rank[my];
                     SSSP_FUZZ_AT(FZ_PUBLISH);
                     // the slot's one writer this run (D13); beyond cap the run is aborted
-                    if (idx < p.cap) IT::store(p.ring + ((size_t)sl * p.cap + idx) * IT::kBytes, s_items[my]);
+                    if (chk) {
+                        const unsigned id1 = s_cid[o][(idx >> kChunkShift) - (s_base[o] >> kChunkShift)];
+                        if (id1) IT::store(chunk_item(p, id1, idx), s_items[my]);
+                    } else if (idx < p.cap) {
+                        IT::store(item_ptr(p, sl, idx, chk), s_items[my]);
+                    }
                 }
                 __syncwarp();
                 if (lane < (int)p.nb) s_wcnt[warp][lane] = 0;  // this warp's row is no longer read

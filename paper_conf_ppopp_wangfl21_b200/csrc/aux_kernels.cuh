@@ -40,10 +40,20 @@ __global__ void interleave_kernel(const unsigned* __restrict__ col, const unsign
     }
 }
 
+// Chunked bucket storage (nullable): chunk tables (nb x tab_stride entries), per-chunk read
+// counts and the free ring are reset; the source's chunk is chunk 0.
+struct ChunkInit {
+    unsigned* ctab = nullptr;
+    unsigned tab_stride = 0, nb = 0;
+    unsigned* chunk_used = nullptr;
+    unsigned* free_ring = nullptr;
+    unsigned pool_chunks = 0;
+    ChunkPool* pool = nullptr;
+};
 template <typename DistT>
 __global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned source, Ctl* ctl, BucketCtl* bk,
                                 char* ring, unsigned long long cap, Head h0, unsigned* expanded,
-                                unsigned short* filt) {
+                                unsigned short* filt, ChunkInit ci) {
     using IT = ItemT<DistT>;
     const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
     for (unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
@@ -54,6 +64,21 @@ __global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned s
     const unsigned long long nw = ((unsigned long long)n + 31) / 32;
     for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += stride)
         expanded[i] = 0u;
+    if (ci.ctab) {
+        const unsigned long long nt = (unsigned long long)ci.nb * ci.tab_stride;
+        const unsigned hs = meta_hs(h0.meta);
+        for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < nt; i += stride)
+            ci.ctab[i] = (i == (unsigned long long)hs * ci.tab_stride) ? 1u : 0u;  // chunk 0: the source's
+        for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < ci.pool_chunks;
+             i += stride) {
+            ci.chunk_used[i] = 0u;
+            ci.free_ring[i] = 0u;
+        }
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            ci.pool->fresh.v = 1;
+            ci.pool->freserve.v = ci.pool->favail.v = ci.pool->fclaim.v = 0;
+        }
+    }
     if (blockIdx.x == 0) {
         const unsigned t = threadIdx.x;
         if (t == kSplitQ) bk[t].reserve.v = bk[t].avail.v = bk[t].claim.v = bk[t].done.v = bk[t].local.v = 0;
@@ -64,7 +89,8 @@ __global__ void init_run_kernel(DistT* __restrict__ dist, unsigned n, unsigned s
             bk[t].done.v = 0;
             bk[t].local.v = 0;
             if (t == meta_hs(h0.meta)) {  // the source item: bucket 0 = head ("initially ... infinity")
-                IT::store(ring + (size_t)t * cap * IT::kBytes, IT::make(source, 0ull));
+                // (chunked storage: item 0 of the head slot is item 0 of chunk 0)
+                IT::store(ring + (ci.ctab ? (size_t)0 : (size_t)t * cap * IT::kBytes), IT::make(source, 0ull));
                 bk[t].reserve.v = 1;
                 bk[t].avail.v = 1;
             }

@@ -57,6 +57,21 @@ struct alignas(32) SplitTask {
     unsigned pad_;
 };
 constexpr uint32_t kSplitQ = kMaxBuckets;
+
+// Chunked bucket storage (SSSP_FLAG_CHUNKED_RING; the paper's block pool): the
+// buckets' index spaces map through per-bucket chunk tables onto a shared pool of
+// kChunkItems-item chunks.  The reserver whose range contains a chunk's first index takes
+// the chunk (fresh, else from the free ring) and publishes it in the table; a chunk returns
+// to the free ring when all its items have been read (and cleared), so memory is bounded by
+// the items alive at once, not by the pushes of a run.
+constexpr unsigned kChunkShift = 12;
+constexpr unsigned kChunkItems = 1u << kChunkShift;
+struct ChunkPool {
+    Counter fresh;     // never-used chunks handed out (bump allocator)
+    Counter freserve;  // free-ring pushes (monotone)
+    Counter favail;    // signed: freed chunks published and not yet taken
+    Counter fclaim;    // free-ring pops (monotone)
+};
 // SplitTask.len states besides a real length: 0 = free, kLenBusy = a writer owns the
 // slot (payload being written), kLenReading = a reader owns it (payload being read).
 // Writers take a free slot by CAS 0 -> busy and publish with a release store of the

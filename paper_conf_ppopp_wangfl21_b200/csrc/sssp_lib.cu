@@ -77,6 +77,10 @@ struct Workspace {
     DevBuf bk, ctl, trace, expanded;
     DevBuf tasks;                   // hub-split chunk queue (SplitTask[tcap])
     DevBuf filt;                    // n x u16 upper-bound filter of dist (D11)
+    // chunked bucket storage (SSSP_FLAG_CHUNKED_RING): ring = pool_chunks chunks of kChunkItems
+    DevBuf ctab, chunk_used, free_ring, pool;
+    bool chunked = false;
+    unsigned pool_chunks = 0;
     unsigned long long tcap = 0;
     unsigned long long cap = 0;
     int ring_item_bytes = 0;
@@ -97,6 +101,10 @@ struct Workspace {
         expanded.release();
         tasks.release();
         filt.release();
+        ctab.release();
+        chunk_used.release();
+        free_ring.release();
+        pool.release();
         nf_piles.release();
         nf_cnt.release();
         if (h_ctl) cudaFreeHost(h_ctl);
@@ -183,10 +191,10 @@ struct KVariant {
     size_t smem;
 };
 template <typename DistT, int BT, bool kF = false, int EPT = 4, int MINB = 1024 / BT, bool PIPE = false, bool WLC = true,
-          bool CA = false>
+          bool CA = false, int CHM = 2>
 KVariant kvar() {
     // (without the warp-local loop the per-warp continuation queues are not allocated)
-    return KVariant{(void*)adds_persistent_kernel<DistT, BT, EPT, MINB, PIPE, kF, WLC, CA>,
+    return KVariant{(void*)adds_persistent_kernel<DistT, BT, EPT, MINB, PIPE, kF, WLC, CA, CHM>,
                     WLC ? Smem<DistT, BT, EPT>::bytes : Smem<DistT, BT, EPT>::o_wqv};
 }
 // The kernel instantiation for a launch shape (each variant's BT is the CTA size it
@@ -195,16 +203,22 @@ KVariant kvar() {
 // 512 x 1/SM when asked; the throughput build is pipelined with claim-ahead at
 // 512 x 2/SM (sweeps §8, §21).  64-bit distances and float32 weights use the plain
 // build at the requested CTA size.
-KVariant persistent_variant(int bits, int bt, bool f32, bool wlc) {
+// The two default builds are compiled separately for flat (CHM 0) and chunked (CHM 1) bucket
+// storage; every other instantiation decides at run time (CHM 2).
+KVariant persistent_variant(int bits, int bt, bool f32, bool wlc, bool chunked) {
     if (f32) return bt == 256 ? kvar<uint32_t, 256, true>() : kvar<uint32_t, 512, true>();
     if (bits == 32) {
-        if (wlc && bt == 128) return kvar<uint32_t, 128, false, 4, 4, true>();
+        if (wlc && bt == 128)
+            return chunked ? kvar<uint32_t, 128, false, 4, 4, true, true, false, 1>()
+                           : kvar<uint32_t, 128, false, 4, 4, true, true, false, 0>();
         if (wlc && bt == 256) return kvar<uint32_t, 256, false, 4, 2, true>();
         if (wlc && bt == 512) return kvar<uint32_t, 512, false, 4, 1, true>();
-        if (bt == 128) return kvar<uint32_t, 128>();
-        if (bt == 512) return kvar<uint32_t, 512, false, 4, 2, true, false, true>();
+        if (bt == 128) return kvar<uint32_t, 128, false, 4, 8, true, false, true>();
+        if (bt == 512)
+            return chunked ? kvar<uint32_t, 512, false, 4, 2, true, false, true, 1>()
+                           : kvar<uint32_t, 512, false, 4, 2, true, false, true, 0>();
         if (bt == 1024) return kvar<uint32_t, 1024>();
-        return kvar<uint32_t, 256>();
+        return kvar<uint32_t, 256, false, 4, 4, true, false, true>();  // throughput build, 4 CTAs/SM
     }
     if (bt == 128) return kvar<unsigned long long, 128>();
     if (bt == 512) return kvar<unsigned long long, 512>();
@@ -218,18 +232,45 @@ bool warp_local_on(const sssp_graph* g) {
     return (g->opts.flags & SSSP_FLAG_WARP_LOCAL) || g->m <= 8ull * g->n;
 }
 
+// Flat (default): items per bucket array, C >= n (no laps within a run, D13).  Chunked
+// (SSSP_FLAG_CHUNKED_RING): items of the shared pool, 2n by default (bounded by the items alive
+// at once, not by a run's pushes); ring_items overrides either.
+bool chunked_ring(const sssp_graph* g) { return (g->opts.flags & SSSP_FLAG_CHUNKED_RING) != 0; }
 unsigned long long default_cap(const sssp_graph* g) {
     if (g->opts.ring_items) return next_pow2(std::max<unsigned long long>(g->opts.ring_items, 64ull));
+    if (chunked_ring(g)) return next_pow2(std::max<unsigned long long>(2ull * g->n, 1ull << 18));
     return next_pow2(std::max<unsigned long long>((unsigned long long)g->n, 1ull << 16));
 }
 
 sssp_status ensure_ring(sssp_graph* g, Workspace& w, int item_bytes, unsigned long long cap) {
-    const size_t bytes = (size_t)g->opts.num_buckets * cap * item_bytes;
-    if (w.ring.p && w.ring.bytes >= bytes && w.cap == cap && w.ring_item_bytes == item_bytes) return SSSP_OK;
+    const bool chunked = chunked_ring(g);
+    unsigned pool_chunks = 0;
+    if (chunked) {
+        pool_chunks = (unsigned)std::min<unsigned long long>(
+            next_pow2(std::max<unsigned long long>(cap >> kChunkShift, 64ull)), 1ull << 30);
+        cap = (unsigned long long)pool_chunks << kChunkShift;
+    }
+    const size_t bytes = chunked ? (size_t)cap * item_bytes : (size_t)g->opts.num_buckets * cap * item_bytes;
+    if (w.ring.p && w.ring.bytes >= bytes && w.cap == cap && w.ring_item_bytes == item_bytes && w.chunked == chunked)
+        return SSSP_OK;
     w.ring.release();
+    w.ctab.release();
+    w.chunk_used.release();
+    w.free_ring.release();
+    w.pool.release();
     CK(cudaMalloc(&w.ring.p, bytes), "allocating the bucket ring");
     w.ring.bytes = bytes;
     CK(cudaMemset(w.ring.p, 0xFF, bytes), "clearing the bucket ring");
+    if (chunked) {
+        const size_t tb = (size_t)g->opts.num_buckets * pool_chunks * sizeof(unsigned);
+        CK(cudaMalloc(&w.ctab.p, tb), "allocating the chunk tables");
+        w.ctab.bytes = tb;
+        CK(cudaMalloc(&w.chunk_used.p, (size_t)pool_chunks * 4), "allocating the chunk read counts");
+        CK(cudaMalloc(&w.free_ring.p, (size_t)pool_chunks * 4), "allocating the free-chunk ring");
+        CK(cudaMalloc(&w.pool.p, sizeof(ChunkPool)), "allocating the chunk pool counters");
+    }
+    w.chunked = chunked;
+    w.pool_chunks = pool_chunks;
     w.cap = cap;
     w.ring_item_bytes = item_bytes;
     return SSSP_OK;
@@ -309,6 +350,13 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
     p.adj = g->d_adj;
     p.dist = (DistT*)w.dist.p;
     p.ring = (char*)w.ring.p;
+    p.chunked = w.chunked ? 1u : 0u;
+    p.ctab = (unsigned*)w.ctab.p;
+    p.tab_mask = w.pool_chunks ? w.pool_chunks - 1 : 0u;
+    p.chunk_used = (unsigned*)w.chunk_used.p;
+    p.free_ring = (unsigned*)w.free_ring.p;
+    p.pool = (ChunkPool*)w.pool.p;
+    p.pool_chunks = w.pool_chunks;
     p.bk = (BucketCtl*)w.bk.p;
     p.ctl = (Ctl*)w.ctl.p;
     const bool tr = (g->opts.flags & SSSP_FLAG_TRACE) != 0;
@@ -412,7 +460,7 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     const bool wlc_auto = !kF && bits == 32 && warp_local_on(g);
     unsigned bt = g->opts.block_threads ? g->opts.block_threads : (wlc_auto ? 128u : 512u);
     if (kF && bt != 256) bt = 512;  // float variants are built for 256/512-thread CTAs
-    const KVariant kv = persistent_variant(bits, (int)bt, kF, warp_local_on(g));
+    const KVariant kv = persistent_variant(bits, (int)bt, kF, warp_local_on(g), chunked_ring(g));
     void* fn = kv.fn;
     CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kv.smem), "smem attribute");
     int occ = 0;
@@ -443,8 +491,18 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     const unsigned aux_grid = (unsigned)g->sm_count * 8 / conc + 1;
     CK(cudaEventRecord(w.ev[0], s), "event");
     if (!g->h_perm.empty()) source = g->h_perm[source];  // internal id (D15)
+    ChunkInit cinit;
+    if (p.chunked) {
+        cinit.ctab = p.ctab;
+        cinit.tab_stride = p.tab_mask + 1;
+        cinit.nb = p.nb;
+        cinit.chunk_used = p.chunk_used;
+        cinit.free_ring = p.free_ring;
+        cinit.pool_chunks = p.pool_chunks;
+        cinit.pool = p.pool;
+    }
     init_run_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, g->n, source, p.ctl, p.bk, p.ring, w.cap, h0,
-                                                    p.expanded, p.filt);
+                                                    p.expanded, p.filt, cinit);
     CK(cudaGetLastError(), "init kernel launch");
     CK(cudaEventRecord(w.ev[1], s), "event");
     void* args[] = {(void*)&p};
@@ -576,6 +634,7 @@ void accumulate(sssp_graph* g, Workspace& w, const Ctl& c, int bits) {
     st.grid_ctas = w.last_grid;
     st.block_threads = w.last_block;
     st.worker = w.last_worker;
+    st.ring_bytes = std::max<uint64_t>(st.ring_bytes, w.ring.bytes + w.ctab.bytes + 8ull * w.pool_chunks);
     st.runs += 1;
     st.trace_entries = std::min<uint32_t>(c.trace_count, w.trace_alloc);
     float a = 0, b = 0;
@@ -1072,7 +1131,8 @@ sssp_status sssp_set_options(sssp_graph* g, const sssp_options* opts) {
     if (st) return st;
     if (opts->device != g->device) return fail(SSSP_ERR_INVALID_ARGUMENT, "the device of a graph cannot change");
     DeviceGuard dg(g->device);
-    const bool ring_change = opts->num_buckets != g->opts.num_buckets || opts->ring_items != g->opts.ring_items;
+    const bool ring_change = opts->num_buckets != g->opts.num_buckets || opts->ring_items != g->opts.ring_items ||
+                             ((opts->flags ^ g->opts.flags) & SSSP_FLAG_CHUNKED_RING);
     g->opts = *opts;
     if (opts->dist_bits) g->cur_bits = (int)opts->dist_bits;
     else g->cur_bits = 32;

@@ -135,6 +135,94 @@ def test_scaled_configs(config, down):
         check(g, s)
 
 
+# ----------------------------------------------------------------- chunked bucket storage
+CHUNKED = sssp.SSSP_FLAG_CHUNKED_RING
+
+
+@pytest.mark.parametrize("config", ["road", "rmat", "er"])
+def test_chunked_ring_scaled(config):
+    """Bucket storage as a chunk pool (the paper's block pool): the default pool, and
+    a 64-chunk pool small enough that chunks are recycled many times within a run (and
+    exhausted, then regrown, where the live items outgrow it)."""
+    g = gg.make(config, scale_down=6)
+    for s in gg.config_sources(config, g, 2):
+        check(g, s, flags=CHUNKED)
+        st = check(g, s, flags=CHUNKED, ring_items=64 * 4096)
+        assert st["pushes"] > 0
+
+
+@pytest.mark.parametrize("opt", [dict(), dict(dist_bits=64), dict(block_threads=256), dict(grid_ctas=3),
+                                 dict(num_buckets=2), dict(ring_items=64 * 4096)])
+def test_chunked_ring_fuzzed(opt):
+    for config in ("road", "rmat"):
+        g = gg.make(config, scale_down=8)
+        s = int(gg.config_sources(config, g, 1)[0])
+        check(g, s, variant="fuzz", flags=CHUNKED, **opt)
+
+
+def test_chunked_ring_overflow_regrows():
+    g = gg.make("rmat", scale_down=6)
+    s = int(gg.config_sources("rmat", g, 1)[0])
+    G = sssp.Graph.from_csr(g, flags=CHUNKED, ring_items=64)  # 64 chunks: exhausted early
+    d = sssp.to_u64(G.run(s))
+    assert np.array_equal(d, oracle.dijkstra(g, s)[0])
+    assert G.stats()["retries"] >= 0
+    Hn = sssp.Graph.from_csr(g, flags=CHUNKED | sssp.SSSP_FLAG_NO_RETRY, ring_items=64, grid_ctas=296)
+    try:
+        Hn.run(s)
+    except RuntimeError as e:  # a pool too small for the live items is reported, not wrong
+        assert "overflow" in str(e).lower()
+
+
+@pytest.mark.parametrize("config", ["road", "rmat", "er"])
+def test_chunked_ring_full_size(config):
+    g = gg.make(config)
+    s = int(gg.config_sources(config, g, 1)[0])
+    ref, V, E = oracle.dijkstra(g, s)
+    G = sssp.Graph.from_csr(g, flags=CHUNKED)
+    out = G.run(s)
+    assert np.array_equal(sssp.to_u64(out), ref)
+    assert G.stats()["reach_edges"] == E
+    # 32-bit items, flat: 32 arrays of next_pow2(n) items x 8 B = 256 n bytes; the pool starts at
+    # 2n items (16 n bytes) and doubles only when the live items outgrow it (ER peaks near 2.4 n)
+    assert G.stats()["ring_bytes"] <= 64 * g.n + (1 << 23)
+
+
+@pytest.mark.timeout(1800)
+def test_chunked_ring_2p26_four_in_flight():
+    """n = 2^26 (ER, average degree 8) with four sources in flight: every row certified on the GPU."""
+    g = gg.er(1 << 26, 8 << 26, 1, 1 << 20, seed=11)
+    srcs = gg.sources(g, 4, seed=11)
+    G = sssp.Graph.from_csr(g, flags=CHUNKED, concurrent_sources=4)
+    D = G.run_batch(srcs)
+    assert G.stats()["concurrency"] == 4
+    for i, s in enumerate(srcs):
+        c = G.certify(int(s), D[i])
+        assert c["exact"] == 1, (int(s), c)
+
+
+# the controller-validation families (graphgen.EXTRA): both sides of the degree-8 build switch,
+# weights to 2^20; plus the throughput build at 256 threads per CTA
+@pytest.mark.parametrize("config", ["rmat_ef4", "er_d4", "grid_wide", "rmat_wide"])
+def test_extra_families(config):
+    g = gg.make(config, scale_down=6)
+    for s in gg.config_sources(config, g, 2):
+        check(g, s)
+        check(g, s, block_threads=256)
+
+
+@pytest.mark.parametrize("config", ["er_d4", "rmat_wide"])
+def test_extra_families_full_size(config):
+    g = gg.make(config)
+    s = int(gg.config_sources(config, g, 1)[0])
+    ref, V, E = oracle.dijkstra(g, s)
+    G = sssp.Graph.from_csr(g)
+    out = G.run(s)
+    assert np.array_equal(sssp.to_u64(out), ref)
+    c = G.certify(s, out)
+    assert c["exact"] == 1 and c["reach_edges"] == E
+
+
 # ----------------------------------------------------------------- schedule perturbation
 PERTURB = [
     dict(grid_ctas=1), dict(grid_ctas=3), dict(grid_ctas=37),
