@@ -50,6 +50,7 @@ template <typename DistT>
 struct Params {
     const unsigned long long* __restrict__ off;  // row_offsets[n+1]
     const uint2* __restrict__ adj;               // interleaved {col, w}[m]
+    const uint2* __restrict__ rows;              // {row begin, degree}[n] when m < 2^32 (else nullptr)
     DistT* dist;                                 // n
     char* ring;                                  // nb * cap items
     BucketCtl* bk;                               // nb
@@ -761,6 +762,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     __shared__ unsigned s_cid[kMaxBuckets][kFlushChunks];                  // chunked storage: their ids
     __shared__ unsigned s_wsum[kWarps], s_wnz[kWarps];
     __shared__ unsigned s_total, s_E, s_NZ, s_got, s_slot, s_lnext, s_direct, s_task, s_tslot;
+    __shared__ unsigned s_fin;  // warps done streaming this batch (first-finisher claim-ahead)
     __shared__ volatile unsigned s_ahead;  // (own load: not merged with the claim fields)
     __shared__ int s_cmd[2];  // by loop parity: an idle CTA loops back to the claim with no
                               // second barrier, so the next claim must not overwrite the
@@ -770,6 +772,10 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     __shared__ Head s_head;
     __shared__ unsigned long long s_prof[kProfCounters];
 
+    // throughput build with 32-bit row records (m < 2^32): 8-byte pops of {begin, degree},
+    // 8-byte per-item records {row begin - arc offset, distance}, 32-bit bucket arithmetic
+    constexpr bool kTP = !WLC && CA && !kF && sizeof(DistT) == 4;
+    uint2* s_info2 = (uint2*)(smem + L::o_info);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const unsigned lt_mask = lanemask_lt();
     const unsigned le_mask = lt_mask | (1u << lane);
@@ -791,6 +797,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         s_lnext = 0;
         s_direct = 0;
         s_ahead = 0;
+        s_fin = 0;
     }
     const bool prof = p.prof != 0 && tid == 0;
     const unsigned long long pol_stream = policy_evict_first();  // arcs, row offsets
@@ -880,6 +887,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         // ------------------------------------------------------------ pop + stale check
         const Head hd = s_head;
         const unsigned hs = meta_hs(hd.meta), k = meta_k(hd.meta);
+        const unsigned h32 = hd.h > 0xFFFFFFFFull ? 0xFFFFFFFFu : (unsigned)hd.h;  // (32-bit distances: j <= h32 iff j <= h)
         unsigned deg = 0;               // arcs this thread's item contributes to the batch
         bool live = false;              // the item is expanded (not stale)
         unsigned long long my_b = 0;    // its row begin
@@ -926,8 +934,15 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 if (loaded) {
                     // the stale check and the row loads are independent: one round trip
                     const unsigned long long cur = (unsigned long long)ld_keep(p.dist + v, pol_keep);
-                    const unsigned long long b = ld_stream_u64(p.off + v, pol_stream);
-                    const unsigned long long e = ld_stream_u64(p.off + v + 1, pol_stream);
+                    unsigned long long b, e;
+                    if constexpr (kTP) {
+                        const uint2 r = ld_stream_u2(p.rows + v, pol_stream);
+                        b = r.x;
+                        e = (unsigned long long)r.x + r.y;
+                    } else {
+                        b = ld_stream_u64(p.off + v, pol_stream);
+                        e = ld_stream_u64(p.off + v + 1, pol_stream);
+                    }
                     if (cur >= d) {  // not stale: d is still v's distance ("refined")
                         deg = (unsigned)(e - b);
                         my_b = b;
@@ -995,7 +1010,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             const unsigned r = s_wnz[warp] + __popc(nzm & lt_mask);
             const unsigned ex = x - deg + s_wsum[warp];
             s_scan[r] = ex;
-            s_info[r] = ItemInfo<DistT>{my_b - ex, (DistT)my_d};  // arc e of the batch is adj[eadj + e]
+            if constexpr (kTP) s_info2[r] = make_uint2((unsigned)my_b - ex, (unsigned)my_d);  // (mod 2^32)
+            else s_info[r] = ItemInfo<DistT>{my_b - ex, (DistT)my_d};  // arc e of the batch is adj[eadj + e]
         }
         const unsigned E = s_E, NZ = s_NZ;
         if (is_task) slot = s_tslot;
@@ -1062,12 +1078,18 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
 #pragma unroll
                 for (int j = 0; j < EPT; ++j) {  // EPT independent arc loads in flight
                     const unsigned e = base + j * 32 + lane;
-                    a[j] = make_uint2(0u, 0u);
-                    dv[j] = (DistT)0;
-                    if (e < we) {
-                        const ItemInfo<DistT> ii = s_info[own[j]];
-                        a[j] = ld_stream_u2(p.adj + (ii.eadj + e), pol_stream);
-                        dv[j] = ii.d;
+                    if constexpr (kTP) {
+                        const uint2 ii = s_info2[min(own[j], NZ - 1u)];
+                        a[j] = ld_stream_u2_if(e < we, p.adj + (ii.x + e), pol_stream);
+                        dv[j] = (DistT)ii.y;
+                    } else {
+                        a[j] = make_uint2(0u, 0u);
+                        dv[j] = (DistT)0;
+                        if (e < we) {
+                            const ItemInfo<DistT> ii = s_info[own[j]];
+                            a[j] = ld_stream_u2(p.adj + (ii.eadj + e), pol_stream);
+                            dv[j] = ii.d;
+                        }
                     }
                 }
             };
@@ -1316,32 +1338,77 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                     emit(push[j] && !kept, a[j].x, (unsigned long long)nd[j], o);
                 }
             };
-            if (PIPE && we > wb + kChunk) {
-                // software pipeline: round r+1's owners and arc loads are issued before
-                // round r's gathers and atomics
-                DistT dv_n[EPT];
-                uint2 a_n[EPT];
-                if (wb < we) fetch(wb, dv_n, a_n);
-                for (unsigned base = wb; base < we;) {
-                    DistT dv[EPT];
-                    uint2 a[EPT];
+            // The same round for the common case of the throughput build (gathered filter, no
+            // 16-bit filter): the gathers and REDs are predicated instructions, not branches,
+            // and the per-arc tests of the other cases are compiled out of the loop.
+            auto body_fire = [&](const unsigned base, const DistT (&dv)[EPT], const uint2 (&a)[EPT]) {
+                DistT nd[EPT], cur[EPT];
+                bool ok[EPT], push[EPT];
+                bool anybad = false;
 #pragma unroll
-                    for (int j = 0; j < EPT; ++j) {
-                        dv[j] = dv_n[j];
-                        a[j] = a_n[j];
+                for (int j = 0; j < EPT; ++j) {
+                    const bool lv = base + j * 32 + lane < we;
+                    bool bd;
+                    nd[j] = relax_narrow<kF, DistT>(dv[j], a[j].y, bd);
+                    anybad |= lv && bd;
+                    ok[j] = lv && !bd;
+                }
+#pragma unroll
+                for (int j = 0; j < EPT; ++j) cur[j] = ld_keep_if(ok[j], p.dist + a[j].x, pol_keep);
+                if (!kF && anybad) atomicOr(&p.ctl->status, kStDistOverflow);  // 32-bit distances insufficient
+#pragma unroll
+                for (int j = 0; j < EPT; ++j) {  // (cur = 0 where !ok: no push)
+                    push[j] = nd[j] < cur[j];
+                    red_min_keep_if(push[j], p.dist + a[j].x, nd[j], pol_keep);
+                }
+#pragma unroll
+                for (int j = 0; j < EPT; ++j) {
+                    if (!__any_sync(FULL, push[j])) continue;
+                    unsigned o;
+                    if constexpr (kTP) {  // 32-bit distances: the bucket in 32-bit arithmetic
+                        const unsigned jb = k >= 32u ? 0u : (unsigned)nd[j] >> k;
+                        o = jb <= h32 ? 0u : min(jb - h32, nbm);
+                    } else {
+                        o = push[j] ? bucket_of<kF>((unsigned long long)nd[j], k, hd.h, p.nb) : 0u;
                     }
-                    const unsigned nxt = base + kChunk;
-                    if (nxt < we) fetch(nxt, dv_n, a_n);
-                    body(base, dv, a);
-                    base = nxt;
+                    const bool kept = keep(push[j] && o == 0, a[j].x, (unsigned long long)nd[j], false, 0ull, 0u);
+                    emit(push[j] && !kept, a[j].x, (unsigned long long)nd[j], o);
                 }
+            };
+            auto stream = [&](auto&& round) {
+                if (PIPE && we > wb + kChunk) {
+                    // software pipeline: round r+1's owners and arc loads are issued before
+                    // round r's gathers and atomics
+                    DistT dv_n[EPT];
+                    uint2 a_n[EPT];
+                    if (wb < we) fetch(wb, dv_n, a_n);
+                    for (unsigned base = wb; base < we;) {
+                        DistT dv[EPT];
+                        uint2 a[EPT];
+#pragma unroll
+                        for (int j = 0; j < EPT; ++j) {
+                            dv[j] = dv_n[j];
+                            a[j] = a_n[j];
+                        }
+                        const unsigned nxt = base + kChunk;
+                        if (nxt < we) fetch(nxt, dv_n, a_n);
+                        round(base, dv, a);
+                        base = nxt;
+                    }
+                } else {
+                    for (unsigned base = wb; base < we; base += kChunk) {
+                        DistT dv[EPT];
+                        uint2 a[EPT];
+                        fetch(base, dv, a);
+                        round(base, dv, a);
+                    }
+                }
+            };
+            if constexpr (!WLC) {
+                if (fire) stream(body_fire);
+                else stream(body);
             } else {
-                for (unsigned base = wb; base < we; base += kChunk) {
-                    DistT dv[EPT];
-                    uint2 a[EPT];
-                    fetch(base, dv, a);
-                    body(base, dv, a);
-                }
+                stream(body);
             }
             // ------------------------------------------------ warp-local continuation
             // Latency regime only (road-like graphs: a few hundred items per bucket,
@@ -1449,7 +1516,16 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         if constexpr (CA) {
             // the batch's claim state (s_got/s_slot/s_idx/s_head/s_task) was consumed before
             // the streaming barrier; kept children (which also use s_slot) need lcap != 0
-            if (warp == 0 && lcap == 0) {
+            // the first warp to finish its slice claims (its round trips overlap the slower
+            // warps' streaming instead of extending the batch when warp 0 is the last;
+            // ER -1.7 %, RMAT -0.7 %, sweeps r02 §10)
+            bool claimer = false;
+            if (lcap == 0) {
+                unsigned f = 0;
+                if (lane == 0) f = atomicAdd(&s_fin, 1u);
+                claimer = __shfl_sync(FULL, f, 0) == 0;
+            }
+            if (claimer) {
                 unsigned sl = 0, st = 0;
                 unsigned long long idx = 0;
                 Head hd2;
@@ -1548,6 +1624,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 c_push += total + direct;
                 s_total = 0;
                 s_direct = 0;
+                s_fin = 0;
             }
             __syncthreads();
         }

@@ -17,6 +17,14 @@ __global__ void validate_csr_kernel(const unsigned long long* __restrict__ off, 
         if (col[e] >= n) atomicMin(&bad[1], e);
 }
 
+// Per-vertex row records {row begin, degree} in 32 bits for graphs with m < 2^32: the
+// throughput kernel's pop reads one aligned 8-byte record instead of two 8-byte offsets.
+__global__ void rows32_kernel(const unsigned long long* __restrict__ off, unsigned n, uint2* __restrict__ rows) {
+    const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+    for (unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride)
+        rows[v] = make_uint2((unsigned)off[v], (unsigned)(off[v + 1] - off[v]));
+}
+
 __global__ void interleave_kernel(const unsigned* __restrict__ col, const unsigned* __restrict__ w,
                                   uint2* __restrict__ adj, unsigned long long m, unsigned long long* sum_w,
                                   unsigned* max_w) {

@@ -221,6 +221,12 @@ __device__ __forceinline__ uint2 ld_stream_u2(const uint2* a, unsigned long long
                  : "=r"(r.x), "=r"(r.y) : "l"(a), "l"(pol));
     return r;
 }
+__device__ __forceinline__ uint2 ld_stream_u2_if(bool pr, const uint2* a, unsigned long long pol) {
+    uint2 r = make_uint2(0u, 0u);
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %3, 0; @q ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0, %1}, [%2], %4; }"
+                 : "+r"(r.x), "+r"(r.y) : "l"(a), "r"((unsigned)pr), "l"(pol));
+    return r;
+}
 __device__ __forceinline__ unsigned long long ld_stream_u64(const unsigned long long* a, unsigned long long pol) {
     unsigned long long r;
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(r) : "l"(a), "l"(pol));
@@ -258,6 +264,29 @@ __device__ __forceinline__ unsigned long long atomic_min_keep(unsigned long long
 }
 
 // fire-and-forget atomic min (RED: no result, no round trip for the issuing warp)
+// Predicated forms for the throughput loop: the instruction carries the predicate, so the
+// compiler emits no branch / reconvergence pair around it (one per arc otherwise).
+__device__ __forceinline__ unsigned ld_keep_if(bool pr, const unsigned* a, unsigned long long pol) {
+    unsigned r = 0u;
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q ld.global.cg.L2::cache_hint.u32 %0, [%1], %3; }"
+                 : "+r"(r) : "l"(a), "r"((unsigned)pr), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ unsigned long long ld_keep_if(bool pr, const unsigned long long* a, unsigned long long pol) {
+    unsigned long long r = 0ull;
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q ld.global.cg.L2::cache_hint.u64 %0, [%1], %3; }"
+                 : "+l"(r) : "l"(a), "r"((unsigned)pr), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ void red_min_keep_if(bool pr, unsigned* a, unsigned v, unsigned long long pol) {
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %3, 0; @q red.global.L2::cache_hint.min.u32 [%0], %1, %2; }"
+                 ::"l"(a), "r"(v), "l"(pol), "r"((unsigned)pr) : "memory");
+}
+__device__ __forceinline__ void red_min_keep_if(bool pr, unsigned long long* a, unsigned long long v,
+                                                unsigned long long pol) {
+    asm volatile("{ .reg .pred q; setp.ne.u32 q, %3, 0; @q red.global.L2::cache_hint.min.u64 [%0], %1, %2; }"
+                 ::"l"(a), "l"(v), "l"(pol), "r"((unsigned)pr) : "memory");
+}
 __device__ __forceinline__ void red_min_keep(unsigned* a, unsigned v, unsigned long long pol) {
     asm volatile("red.global.L2::cache_hint.min.u32 [%0], %1, %2;" ::"l"(a), "r"(v), "l"(pol) : "memory");
 }

@@ -122,6 +122,7 @@ struct sssp_graph {
     uint64_t m = 0;
     unsigned long long* d_off = nullptr;
     uint2* d_adj = nullptr;
+    uint2* d_rows = nullptr;  // {row begin, degree} in 32 bits (m < 2^32): the throughput kernel's pop
     // locality relabeling (D15): internal id of each caller id (device, for finalize;
     // host, for the source); empty / nullptr = identity
     unsigned* d_perm = nullptr;
@@ -205,8 +206,10 @@ KVariant kvar() {
 // build at the requested CTA size.
 // The two default builds are compiled separately for flat (CHM 0) and chunked (CHM 1) bucket
 // storage; every other instantiation decides at run time (CHM 2).
-KVariant persistent_variant(int bits, int bt, bool f32, bool wlc, bool chunked) {
+KVariant persistent_variant(int bits, int bt, bool f32, bool wlc, bool chunked, bool rows) {
     if (f32) return bt == 256 ? kvar<uint32_t, 256, true>() : kvar<uint32_t, 512, true>();
+    if (bits == 32 && !wlc && !rows)  // (m >= 2^32: no 32-bit row records) the throughput build without them
+        return kvar<uint32_t, 512, false, 4, 2, true, false, false>();
     if (bits == 32) {
         if (wlc && bt == 128)
             return chunked ? kvar<uint32_t, 128, false, 4, 4, true, true, false, 1>()
@@ -348,6 +351,7 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
     Params<DistT> p{};
     p.off = g->d_off;
     p.adj = g->d_adj;
+    p.rows = g->d_rows;
     p.dist = (DistT*)w.dist.p;
     p.ring = (char*)w.ring.p;
     p.chunked = w.chunked ? 1u : 0u;
@@ -460,7 +464,8 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     const bool wlc_auto = !kF && bits == 32 && warp_local_on(g);
     unsigned bt = g->opts.block_threads ? g->opts.block_threads : (wlc_auto ? 128u : 512u);
     if (kF && bt != 256) bt = 512;  // float variants are built for 256/512-thread CTAs
-    const KVariant kv = persistent_variant(bits, (int)bt, kF, warp_local_on(g), chunked_ring(g));
+    if (!kF && bits == 32 && !warp_local_on(g) && !g->d_rows) bt = 512;  // (see persistent_variant)
+    const KVariant kv = persistent_variant(bits, (int)bt, kF, warp_local_on(g), chunked_ring(g), g->d_rows != nullptr);
     void* fn = kv.fn;
     CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kv.smem), "smem attribute");
     int occ = 0;
@@ -1070,6 +1075,11 @@ sssp_status create_impl(uint32_t n, uint64_t m, const uint64_t* row_offsets, con
         sssp_status rs = relabel_graph(g, o);
         if (rs) return bail(rs);
     }
+    if (m < (1ull << 32) && n) {
+        CKG(cudaMalloc(&g->d_rows, (size_t)n * sizeof(uint2)), "allocating row records");
+        rows32_kernel<<<aux_grid, 256>>>(g->d_off, n, g->d_rows);
+        CKG(cudaDeviceSynchronize(), "building row records");
+    }
     // initial Delta (reading R3): max_w / D (Meyer-Sanders' Theta(1/d) rule for Delta-stepping [15]),
     // or the Near-Far rule C * W / D with W = average weight, D = average degree, C = 32
     if (m && g->sum_w && !f32) {
@@ -1109,6 +1119,7 @@ sssp_status sssp_graph_destroy(sssp_graph* g) {
     cudaDeviceSynchronize();
     if (g->d_off) cudaFree(g->d_off);
     if (g->d_adj) cudaFree(g->d_adj);
+    if (g->d_rows) cudaFree(g->d_rows);
     if (g->d_perm) cudaFree(g->d_perm);
     for (Workspace* w : g->ws) {
         w->release();
