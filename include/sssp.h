@@ -146,7 +146,8 @@ typedef struct sssp_options {
     uint32_t flags;            /* SSSP_FLAG_* */
     uint32_t block_threads;    /* worker CTA size: 0 = auto (512; 128 on road-like graphs), else 128/256/512/1024 */
     uint32_t grid_ctas;        /* 0 = every co-resident CTA; else at most this many CTAs */
-    uint32_t batch_min;        /* minimum items a CTA claims when enough are available; 0 = auto */
+    uint32_t batch_min;        /* minimum items a CTA claims when enough are available; 0 = auto
+                                  (256 on the throughput build, 32 on road-like graphs) */
     uint32_t timeout_ms;       /* device watchdog (globaltimer); 0 = default 60000 */
     uint32_t trace_capacity;   /* trace ring entries when SSSP_FLAG_TRACE; 0 = 65536 */
     uint32_t active_init;      /* initial number of active (claimable) buckets; 0 = auto: 4 when

@@ -461,17 +461,24 @@ __device__ __forceinline__ unsigned short filt_enc(unsigned long long x, unsigne
 // they are the unfinished rest of an already-claimed item, usually of the head
 // bucket, which cannot complete before they do.  A chunk claim returns 1 with
 // o_task set and o_idx = the chunk's queue index.
-template <typename DistT, int BT>
+template <typename DistT, int BT, bool kAllGates>
 __device__ unsigned claim_batch(const Params<DistT>& p, int lane, unsigned& o_slot, unsigned long long& o_idx,
                                 Head& o_head, unsigned& o_status, bool& o_task) {
     o_task = false;
     const unsigned nbm = p.nb - 1;
     unsigned st = 0;
     Head hd{0ull, 0ull};
+    // throughput build (kAllGates): one round trip for status + head (lane 0) and every ring
+    // slot's avail gate (lane l reads slot l), the active window's gates picked once the head
+    // slot is known (RMAT/ER -1 %); latency build: the active gates after the head (its many
+    // idle pollers reading 32 hot lines each slowed ROAD 31.2 -> 34.1 ms, sweeps r02 §10)
+    long long avs = 0, tv = 0;
     if (lane == 0) {
         st = ld_relaxed_u32(&p.ctl->status);
         hd = ld_head(&p.ctl->head);
     }
+    if (kAllGates && lane < (int)p.nb) avs = (long long)ld_relaxed_u64(&p.bk[lane].avail.v);
+    if (p.split_deg && lane == 31) tv = (long long)ld_relaxed_u64(&p.bk[kSplitQ].avail.v);
     st = __shfl_sync(FULL, st, 0);
     hd.h = __shfl_sync(FULL, hd.h, 0);
     hd.meta = __shfl_sync(FULL, hd.meta, 0);
@@ -479,9 +486,13 @@ __device__ unsigned claim_batch(const Params<DistT>& p, int lane, unsigned& o_sl
     o_head = hd;
     if (st) return 0;
     const unsigned hs = meta_hs(hd.meta), A = meta_A(hd.meta);
-    long long av = 0, tv = 0;
-    if (lane < (int)A) av = (long long)ld_relaxed_u64(&p.bk[(hs + lane) & nbm].avail.v);
-    if (p.split_deg && lane == 31) tv = (long long)ld_relaxed_u64(&p.bk[kSplitQ].avail.v);
+    long long av;
+    if constexpr (kAllGates) {
+        av = __shfl_sync(FULL, avs, (int)((hs + (unsigned)lane) & nbm));
+        if (lane >= (int)A) av = 0;
+    } else {
+        av = lane < (int)A ? (long long)ld_relaxed_u64(&p.bk[(hs + lane) & nbm].avail.v) : 0;
+    }
     if (__shfl_sync(FULL, tv, 31) > 0) {
         unsigned got = 0;
         unsigned long long ix = 0;
@@ -827,7 +838,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 unsigned long long idx = 0;
                 Head hd;
                 bool tk;
-                const unsigned g = claim_batch<DistT, BT>(p, lane, sl, idx, hd, st, tk);
+                const unsigned g = claim_batch<DistT, BT, !WLC>(p, lane, sl, idx, hd, st, tk);
                 if (st) {
                     cmd = CMD_EXIT;
                 } else if (g) {
@@ -1530,7 +1541,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 unsigned long long idx = 0;
                 Head hd2;
                 bool tk;
-                const unsigned g = claim_batch<DistT, BT>(p, lane, sl, idx, hd2, st, tk);
+                const unsigned g = claim_batch<DistT, BT, !WLC>(p, lane, sl, idx, hd2, st, tk);
                 if (lane == 0 && g) {
                     s_got = g;
                     s_slot = sl;

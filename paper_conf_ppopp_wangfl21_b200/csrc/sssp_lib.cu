@@ -380,7 +380,9 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
     p.resident_threads = (unsigned long long)grid * bt;
     const double deg = g->n ? (double)g->m / g->n : 0.0;
     p.avg_deg_x16 = (unsigned)std::min(16.0 * deg + 0.5, 4.0e9);
-    p.batch_min = g->opts.batch_min ? g->opts.batch_min : 32;
+    // auto: 256 on the throughput side (fewer, larger batches: RMAT/ER -1.7 %, sweeps r02 §10),
+    // 32 on road-like graphs (large batches there break the latency regime: ROAD work 70x)
+    p.batch_min = g->opts.batch_min ? g->opts.batch_min : (warp_local_on(g) ? 32u : 256u);
     unsigned sh = 0;
     while ((1u << (sh + 1)) <= grid) ++sh;  // floor(log2 grid)
     p.share_shift = sh > 2 ? sh - 2 : 0;
