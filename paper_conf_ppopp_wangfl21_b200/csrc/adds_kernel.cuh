@@ -798,6 +798,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     const bool track_busy = p.dynamic && p.adapt_active;
     bool busy_cta = false;  // warp 0 lane 0: this CTA is counted in g_busy
     unsigned have_local = 0;  // uniform: items of the next batch already in s_lv/s_ld
+    unsigned kslot = 0;       // their ring slot (the batch's own)
+    __shared__ unsigned s_nf;  // first expansions of this batch (controller), summed per warp
 
     if (tid < (int)kMaxBuckets) s_cnt[tid] = 0;
     for (int i = tid; i < kWarps * (int)kMaxBuckets; i += BT) (&s_wcnt[0][0])[i] = 0;
@@ -809,6 +811,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         s_direct = 0;
         s_ahead = 0;
         s_fin = 0;
+        s_nf = 0;
     }
     const bool prof = p.prof != 0 && tid == 0;
     const unsigned long long pol_stream = policy_evict_first();  // arcs, row offsets
@@ -823,7 +826,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         if (prof) t0 = clock64();
         if (have_local) {
             got = have_local;
-            slot = s_slot;
+            slot = kslot;
             from_ring = false;
         } else if (CA && s_ahead) {  // claimed ahead by warp 0 during the previous batch
             got = s_got;
@@ -968,7 +971,6 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
             }
         }
-        if (tid == 0) s_lnext = 0;
         if (prof) {
             const long long t1 = clock64();
             s_prof[PR_POP] += t1 - t0;
@@ -991,6 +993,8 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             s_wnz[warp] = __popc(nzm);
         }
         const int nlive = __syncthreads_count(live);
+        // (every thread read the last batch's s_lnext before this barrier: no barrier ends a batch)
+        if (tid == 0) s_lnext = 0;
         // chunked storage: this batch's reads (and clears) are complete; count them per chunk
         if (chk && tid == 0 && from_ring && !is_task) chunks_consumed(p, slot, s_idx, got);
         if (warp == 0) {
@@ -1553,91 +1557,92 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
                 }
             }
         }
+        // first expansions of this batch's pops (controller), one shared atomic per warp
         {
-            const bool any_staged = __syncthreads_or(wfill != 0) != 0;
-            unsigned total = 0;
-            if (any_staged) {
-                // ---------------------------------------------------- flush to the ring
-                const long long tf = prof ? clock64() : 0;
-                {
-                    // column scan of s_wcnt over the warps, all warps at once: lanes form
-                    // segments of kWarps (one per bucket), lane w%kWarps = warp w's count;
-                    // the segment's last lane holds the CTA's count for the bucket and
-                    // reserves it (returning atomic: the reserve, which also counts the
-                    // children for termination, precedes this CTA's completion release)
-                    constexpr unsigned kBPW = kWarps >= 32 ? 1u : 32u / kWarps;  // buckets per warp
-                    const unsigned o = (unsigned)warp * kBPW + (unsigned)lane / kWarps;
-                    const unsigned w = (unsigned)lane % kWarps;
-                    const bool mine = o < p.nb;
-                    const unsigned v = mine ? s_wcnt[w][o] : 0u;
-                    unsigned x = v;
+            const unsigned nf = (unsigned)__popc(__ballot_sync(FULL, fbit != 0 && (fword & fbit) == 0));
+            if (lane == 0 && nf) atomicAdd(&s_nf, nf);
+        }
+        // End of batch, three barriers at most: B1 (streaming done: staging, s_lnext, s_nf, the
+        // claim-ahead and the warp-local counters are final), B2 (reserves done), B3 (stores
+        // done).  No barrier closes the batch: warp 0 publishes, completes and runs the
+        // controller while the other warps start the next batch's pop (they meet again at its
+        // first barrier); what they read here was written before B1 and is reset only after
+        // that next barrier (s_lnext) or by thread 0 itself (s_total, s_direct, s_fin, s_nf).
+        const bool any_staged = __syncthreads_or(wfill != 0) != 0;  // B1
+        const unsigned kept = s_lnext < lcap ? s_lnext : lcap;
+        unsigned total = 0;
+        if (any_staged) {
+            // ---------------------------------------------------- flush to the ring
+            const long long tf = prof ? clock64() : 0;
+            {
+                // column scan of s_wcnt over the warps, all warps at once: lanes form
+                // segments of kWarps (one per bucket), lane w%kWarps = warp w's count;
+                // the segment's last lane holds the CTA's count for the bucket and
+                // reserves it (returning atomic: the reserve, which also counts the
+                // children for termination, precedes this CTA's completion release)
+                constexpr unsigned kBPW = kWarps >= 32 ? 1u : 32u / kWarps;  // buckets per warp
+                const unsigned o = (unsigned)warp * kBPW + (unsigned)lane / kWarps;
+                const unsigned w = (unsigned)lane % kWarps;
+                const bool mine = o < p.nb;
+                const unsigned v = mine ? s_wcnt[w][o] : 0u;
+                unsigned x = v;
 #pragma unroll
-                    for (unsigned d = 1; d < (unsigned)kWarps; d <<= 1) {
-                        const unsigned y = __shfl_up_sync(FULL, x, d, kWarps);
-                        if (w >= d) x += y;
-                    }
-                    if (mine) s_wcnt[w][o] = x - v;  // warp w's offset inside the CTA's reservation
-                    if (mine && w == (unsigned)kWarps - 1) {
-                        s_cnt[o] = x;
-                        if (x) {
-                            atomicAdd(&s_total, x);
-                            const unsigned long long b = atomicAdd(&p.bk[(hs + o) & nbm].reserve.v, (unsigned long long)x);
-                            SSSP_FUZZ_AT(FZ_RESERVE);
-                            s_base[o] = b;
-                            if (flat_overflow(p, b, x, chk)) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
-                            chunks_for_range(p, (hs + o) & nbm, b, x, chk);
-                            if (chk) {  // the range's chunks, once, for every store below
-                                for (unsigned q = 0; q < kFlushChunks; ++q) {
-                                    const unsigned long long ci = (b >> kChunkShift) + q;
-                                    s_cid[o][q] = (ci << kChunkShift) < b + x ? chunk_of(p, (hs + o) & nbm, ci << kChunkShift) : 0u;
-                                }
+                for (unsigned d = 1; d < (unsigned)kWarps; d <<= 1) {
+                    const unsigned y = __shfl_up_sync(FULL, x, d, kWarps);
+                    if (w >= d) x += y;
+                }
+                if (mine) s_wcnt[w][o] = x - v;  // warp w's offset inside the CTA's reservation
+                if (mine && w == (unsigned)kWarps - 1) {
+                    s_cnt[o] = x;
+                    if (x) {
+                        atomicAdd(&s_total, x);
+                        const unsigned long long b = atomicAdd(&p.bk[(hs + o) & nbm].reserve.v, (unsigned long long)x);
+                        SSSP_FUZZ_AT(FZ_RESERVE);
+                        s_base[o] = b;
+                        if (flat_overflow(p, b, x, chk)) atomicOr(&p.ctl->status, kStRingOverflow);  // no laps (D13)
+                        chunks_for_range(p, (hs + o) & nbm, b, x, chk);
+                        if (chk) {  // the range's chunks, once, for every store below
+                            for (unsigned q = 0; q < kFlushChunks; ++q) {
+                                const unsigned long long ci = (b >> kChunkShift) + q;
+                                s_cid[o][q] = (ci << kChunkShift) < b + x ? chunk_of(p, (hs + o) & nbm, ci << kChunkShift) : 0u;
                             }
-                            if (p.dynamic && o == nbm) atomicAdd(&p.ctl->g_clip, (unsigned long long)x);
                         }
+                        if (p.dynamic && o == nbm) atomicAdd(&p.ctl->g_clip, (unsigned long long)x);
                     }
-                }
-                __syncthreads();
-                total = s_total;
-                // each warp stores its own segment (coalesced runs per bucket)
-                for (unsigned i = lane; i < wfill; i += 32) {
-                    const unsigned my = (unsigned)warp * kSeg + i;
-                    const unsigned o = s_soff[my];
-                    const unsigned sl = (hs + o) & nbm;
-                    const unsigned long long idx = s_base[o] + s_wcnt[warp][o] + s_rank[my];
-                    SSSP_FUZZ_AT(FZ_PUBLISH);
-                    // the slot's one writer this run (D13); beyond cap the run is aborted
-                    if (chk) {
-                        const unsigned id1 = s_cid[o][(idx >> kChunkShift) - (s_base[o] >> kChunkShift)];
-                        if (id1) IT::store(chunk_item(p, id1, idx), s_items[my]);
-                    } else if (idx < p.cap) {
-                        IT::store(item_ptr(p, sl, idx, chk), s_items[my]);
-                    }
-                }
-                __syncwarp();
-                if (lane < (int)p.nb) s_wcnt[warp][lane] = 0;  // this warp's row is no longer read
-                __syncthreads();
-                if (warp == 0 && lane < (int)p.nb) {
-                    const unsigned c = s_cnt[lane];
-                    if (p.dynamic && lane == 0) atomicAdd(&p.ctl->g_push, (unsigned long long)(total + s_direct));
-                    if (c) {
-                        atomicAdd(&p.bk[(hs + lane) & nbm].avail.v, (unsigned long long)c);  // publish
-                        s_cnt[lane] = 0;
-                    }
-                }
-                if (prof) {
-                    tq += clock64() - tf;
-                    s_prof[PR_N_FLUSH] += 1;
                 }
             }
-            if (tid == 0) {  // (s_direct is read by thread 0 only: it also resets it)
-                const unsigned direct = s_direct;
-                if (!any_staged && p.dynamic && direct) atomicAdd(&p.ctl->g_push, (unsigned long long)direct);
-                c_push += total + direct;
-                s_total = 0;
-                s_direct = 0;
-                s_fin = 0;
+            __syncthreads();  // B2
+            total = s_total;
+            // each warp stores its own segment (coalesced runs per bucket)
+            for (unsigned i = lane; i < wfill; i += 32) {
+                const unsigned my = (unsigned)warp * kSeg + i;
+                const unsigned o = s_soff[my];
+                const unsigned sl = (hs + o) & nbm;
+                const unsigned long long idx = s_base[o] + s_wcnt[warp][o] + s_rank[my];
+                SSSP_FUZZ_AT(FZ_PUBLISH);
+                // the slot's one writer this run (D13); beyond cap the run is aborted
+                if (chk) {
+                    const unsigned id1 = s_cid[o][(idx >> kChunkShift) - (s_base[o] >> kChunkShift)];
+                    if (id1) IT::store(chunk_item(p, id1, idx), s_items[my]);
+                } else if (idx < p.cap) {
+                    IT::store(item_ptr(p, sl, idx, chk), s_items[my]);
+                }
             }
-            __syncthreads();
+            __syncwarp();
+            if (lane < (int)p.nb) s_wcnt[warp][lane] = 0;  // this warp's row is no longer read
+            __syncthreads();  // B3
+            if (warp == 0 && lane < (int)p.nb) {
+                const unsigned c = s_cnt[lane];
+                if (p.dynamic && lane == 0) atomicAdd(&p.ctl->g_push, (unsigned long long)(total + s_direct));
+                if (c) {
+                    atomicAdd(&p.bk[(hs + lane) & nbm].avail.v, (unsigned long long)c);  // publish
+                    s_cnt[lane] = 0;
+                }
+            }
+            if (prof) {
+                tq += clock64() - tf;
+                s_prof[PR_N_FLUSH] += 1;
+            }
         }
         if (prof) {
             const long long t1 = clock64();
@@ -1648,12 +1653,17 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         }
 
         // ------------------------------------------------------------ complete
-        // s_lnext final (also covers the E == 0 case); first expansions for the controller
-        const int nfirst = __syncthreads_count(fbit != 0 && (fword & fbit) == 0);
-        const unsigned kept = s_lnext < lcap ? s_lnext : lcap;
-        // (thread 0 alone reads the warp-local counters: it also resets them below)
-        unsigned w_exp = 0, w_first = 0, w_kept = 0;
+        // (thread 0 alone reads and resets the CTA's shared counters)
+        unsigned w_exp = 0, w_first = 0, w_kept = 0, nfirst = 0;
         if (tid == 0) {
+            const unsigned direct = s_direct;
+            if (!any_staged && p.dynamic && direct) atomicAdd(&p.ctl->g_push, (unsigned long long)direct);
+            c_push += total + direct;
+            s_total = 0;
+            s_direct = 0;
+            s_fin = 0;
+            nfirst = s_nf;
+            s_nf = 0;
             w_exp = s_wst[0];
             w_first = s_wst[1];
             w_kept = s_wst[4];
@@ -1667,13 +1677,13 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             }
             // one atomic: the kept children inherit the parents' accounting; a completion
             // is a release (common.cuh red_release_add_u64): the children's reserve
-            // atomics above are ordered before it by the CTA barrier
+            // atomics (warp flushes before B1, the CTA flush before B2) are ordered before
+            // it by the CTA barriers
             SSSP_FUZZ_AT(FZ_COMPLETE);
             if (got > kept) red_release_add_u64(&p.bk[slot].done.v, (unsigned long long)(got - kept));
             else if (kept > got) atomicAdd(&p.bk[slot].local.v, (unsigned long long)(kept - got));
             c_push += kept;
             c_local += kept;
-            if (kept) s_slot = slot;
         }
         if (p.dynamic && warp == 0) {
             unsigned run_ctl = 0;
@@ -1690,7 +1700,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
             if (__shfl_sync(FULL, run_ctl, 0)) periodic_step<DistT>(p, lane);
         }
         have_local = kept;
-        __syncthreads();
+        kslot = slot;
         if (prof) s_prof[PR_COMPLETE] += clock64() - t0;
     }
 
