@@ -772,7 +772,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     constexpr unsigned kFlushChunks = ((unsigned)kStage + kChunkItems - 1) / kChunkItems + 1;
     __shared__ unsigned s_cid[kMaxBuckets][kFlushChunks];                  // chunked storage: their ids
     __shared__ unsigned s_wsum[kWarps], s_wnz[kWarps];
-    __shared__ unsigned s_total, s_E, s_NZ, s_got, s_slot, s_lnext, s_direct, s_task, s_tslot;
+    __shared__ unsigned s_total, s_got, s_slot, s_lnext, s_direct, s_task, s_tslot;
     __shared__ unsigned s_fin;  // warps done streaming this batch (first-finisher claim-ahead)
     __shared__ volatile unsigned s_ahead;  // (own load: not merged with the claim fields)
     __shared__ int s_cmd[2];  // by loop parity: an idle CTA loops back to the claim with no
@@ -997,38 +997,21 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         if (tid == 0) s_lnext = 0;
         // chunked storage: this batch's reads (and clears) are complete; count them per chunk
         if (chk && tid == 0 && from_ring && !is_task) chunks_consumed(p, slot, s_idx, got);
-        if (warp == 0) {
-            const unsigned ws = lane < kWarps ? s_wsum[lane] : 0;
-            const unsigned wn = lane < kWarps ? s_wnz[lane] : 0;
-            unsigned inc = ws, incn = wn;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const unsigned y = __shfl_up_sync(FULL, inc, o);
-                const unsigned yn = __shfl_up_sync(FULL, incn, o);
-                if (lane >= o) {
-                    inc += y;
-                    incn += yn;
-                }
-            }
-            if (lane < kWarps) {
-                s_wsum[lane] = inc - ws;
-                s_wnz[lane] = incn - wn;
-            }
-            if (lane == kWarps - 1) {
-                s_E = inc;
-                s_NZ = incn;
-                s_scan[incn] = inc;  // sentinel
-            }
-        }
-        __syncthreads();
+        // every warp combines the kWarps warp totals itself (four warp reductions), so no warp
+        // waits on a serial scan by warp 0 and one barrier is saved
+        const unsigned ws = lane < kWarps ? s_wsum[lane] : 0u;
+        const unsigned wn = lane < kWarps ? s_wnz[lane] : 0u;
+        const unsigned E = __reduce_add_sync(FULL, ws), NZ = __reduce_add_sync(FULL, wn);
+        const unsigned wpre = __reduce_add_sync(FULL, lane < warp ? ws : 0u);
+        const unsigned wnpre = __reduce_add_sync(FULL, lane < warp ? wn : 0u);
+        if (tid == 0) s_scan[NZ] = E;  // sentinel
         if (deg > 0) {
-            const unsigned r = s_wnz[warp] + __popc(nzm & lt_mask);
-            const unsigned ex = x - deg + s_wsum[warp];
+            const unsigned r = wnpre + __popc(nzm & lt_mask);
+            const unsigned ex = x - deg + wpre;
             s_scan[r] = ex;
             if constexpr (kTP) s_info2[r] = make_uint2((unsigned)my_b - ex, (unsigned)my_d);  // (mod 2^32)
             else s_info[r] = ItemInfo<DistT>{my_b - ex, (DistT)my_d};  // arc e of the batch is adj[eadj + e]
         }
-        const unsigned E = s_E, NZ = s_NZ;
         if (is_task) slot = s_tslot;
         const int nexp = is_task ? 0 : nlive;  // a chunk is not a vertex expansion
         if (tid == 0) {
