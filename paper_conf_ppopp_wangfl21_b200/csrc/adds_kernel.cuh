@@ -823,12 +823,14 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
     for (;;) {
         unsigned got, slot;
         bool from_ring, is_task = false;
+        bool ahead = false;  // this batch is the one claimed ahead
         if (prof) t0 = clock64();
         if (have_local) {
             got = have_local;
             slot = kslot;
             from_ring = false;
-        } else if (CA && s_ahead) {  // claimed ahead by warp 0 during the previous batch
+        } else if (CA && s_ahead) {  // claimed ahead during a previous batch
+            ahead = true;
             got = s_got;
             slot = s_slot;
             from_ring = true;
@@ -1028,7 +1030,7 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         }
 
         __syncthreads();  // publishes s_scan / s_info
-        if (CA && tid == 0) s_ahead = 0;  // every thread has read it (loop top)
+        if (CA && ahead && tid == 0) s_ahead = 0;  // every thread has read it (loop top)
         unsigned wfill = 0;  // warp-uniform: items staged in this warp's segment
         // ---------------------------------------------------- stream the batch's arcs
         // Warp w owns a contiguous slice of the batch's arc space and streams through
@@ -1513,12 +1515,15 @@ __global__ void __launch_bounds__(BT, MINB) adds_persistent_kernel(const Params<
         }
         if constexpr (CA) {
             // the batch's claim state (s_got/s_slot/s_idx/s_head/s_task) was consumed before
-            // the streaming barrier; kept children (which also use s_slot) need lcap != 0
+            // the streaming barrier
             // the first warp to finish its slice claims (its round trips overlap the slower
             // warps' streaming instead of extending the batch when warp 0 is the last;
             // ER -1.7 %, RMAT -0.7 %, sweeps r02 §10)
+            // A batch that keeps children (lcap != 0) claims ahead too: its kept children run
+            // first (loop top), the claimed batch waits in s_got.. until no local batch is left
+            // (one claim ahead at most; kept children use their own slot, kslot)
             bool claimer = false;
-            if (lcap == 0) {
+            if (!s_ahead) {
                 unsigned f = 0;
                 if (lane == 0) f = atomicAdd(&s_fin, 1u);
                 claimer = __shfl_sync(FULL, f, 0) == 0;
