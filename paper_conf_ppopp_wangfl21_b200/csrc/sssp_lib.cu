@@ -217,9 +217,15 @@ KVariant persistent_variant(int bits, int bt, bool f32, bool wlc, bool chunked, 
         if (wlc && bt == 256) return kvar<uint32_t, 256, false, 4, 2, true>();
         if (wlc && bt == 512) return kvar<uint32_t, 512, false, 4, 1, true>();
         if (bt == 128) return kvar<uint32_t, 128, false, 4, 8, true, false, true>();
+// (throughput build: 3 arcs per thread per round -- fewer live registers at the 64-register
+// budget than 4: config 5 -3 %, ER -0.5 %; 2 is faster on config 5 but +1.5 % on ER, and 5-6
+// spill: sweeps r02 §10)
+#ifndef SSSP_TP_EPT
+#define SSSP_TP_EPT 3
+#endif
         if (bt == 512)
-            return chunked ? kvar<uint32_t, 512, false, 4, 2, true, false, true, 1>()
-                           : kvar<uint32_t, 512, false, 4, 2, true, false, true, 0>();
+            return chunked ? kvar<uint32_t, 512, false, SSSP_TP_EPT, 2, true, false, true, 1>()
+                           : kvar<uint32_t, 512, false, SSSP_TP_EPT, 2, true, false, true, 0>();
         if (bt == 1024) return kvar<uint32_t, 1024>();
         return kvar<uint32_t, 256, false, 4, 4, true, false, true>();  // throughput build, 4 CTAs/SM
     }
