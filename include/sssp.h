@@ -89,6 +89,10 @@ typedef enum sssp_status {
                                         block pool): memory bounded by the items alive at
                                         once (default pool 2n items, grown x2 on exhaustion) instead of
                                         one no-lap array of >= n items per bucket (32n items) */
+#define SSSP_FLAG_WIDE_ROWS 0x4000u /* the throughput build reads the 64-bit row offsets instead of its
+                                       32-bit row records {begin, degree} -- the path graphs with
+                                       m >= 2^32 take (no records are built for them); for tests and
+                                       ablations */
 #define SSSP_FLAG_L2_PERSIST 0x20u /* reserve the L2 persisting set-aside for dist (raises the device-wide
                                      cudaLimitPersistingL2CacheSize to min(dist bytes, maximum)) and mark
                                      dist accesses evict_last.  Off by default: measured on B200

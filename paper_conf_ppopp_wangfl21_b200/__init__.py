@@ -36,6 +36,7 @@ SSSP_FLAG_L2_PERSIST = 0x20
 SSSP_FLAG_ADAPT_ACTIVE = 0x40  # (default since round 2)
 SSSP_FLAG_FIXED_ACTIVE = 0x1000
 SSSP_FLAG_CHUNKED_RING = 0x2000
+SSSP_FLAG_WIDE_ROWS = 0x4000
 SSSP_FLAG_NO_WARP_LOCAL = 0x80
 SSSP_FLAG_WARP_LOCAL = 0x100
 SSSP_FLAG_FILTER16 = 0x200

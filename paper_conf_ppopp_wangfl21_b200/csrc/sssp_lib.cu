@@ -357,7 +357,7 @@ Params<DistT> make_params(sssp_graph* g, Workspace& w, unsigned grid, unsigned b
     Params<DistT> p{};
     p.off = g->d_off;
     p.adj = g->d_adj;
-    p.rows = g->d_rows;
+    p.rows = (g->opts.flags & SSSP_FLAG_WIDE_ROWS) ? nullptr : g->d_rows;
     p.dist = (DistT*)w.dist.p;
     p.ring = (char*)w.ring.p;
     p.chunked = w.chunked ? 1u : 0u;
@@ -472,8 +472,9 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
     const bool wlc_auto = !kF && bits == 32 && warp_local_on(g);
     unsigned bt = g->opts.block_threads ? g->opts.block_threads : (wlc_auto ? 128u : 512u);
     if (kF && bt != 256) bt = 512;  // float variants are built for 256/512-thread CTAs
-    if (!kF && bits == 32 && !warp_local_on(g) && !g->d_rows) bt = 512;  // (see persistent_variant)
-    const KVariant kv = persistent_variant(bits, (int)bt, kF, warp_local_on(g), chunked_ring(g), g->d_rows != nullptr);
+    const bool rows32 = g->d_rows && !(g->opts.flags & SSSP_FLAG_WIDE_ROWS);
+    if (!kF && bits == 32 && !warp_local_on(g) && !rows32) bt = 512;  // (see persistent_variant)
+    const KVariant kv = persistent_variant(bits, (int)bt, kF, warp_local_on(g), chunked_ring(g), rows32);
     void* fn = kv.fn;
     CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kv.smem), "smem attribute");
     int occ = 0;

@@ -250,6 +250,9 @@ PERTURB = [
     dict(flags=sssp.SSSP_FLAG_RELABEL), dict(flags=sssp.SSSP_FLAG_NO_RELABEL),
     dict(flags=sssp.SSSP_FLAG_RELABEL, dist_bits=64),
     dict(flags=sssp.SSSP_FLAG_RELABEL, algorithm=sssp.SSSP_ALGO_NEAR_FAR),
+    # the throughput build on 64-bit row offsets (the m >= 2^32 path), with 256-thread CTAs and hub splits
+    dict(flags=sssp.SSSP_FLAG_WIDE_ROWS), dict(flags=sssp.SSSP_FLAG_WIDE_ROWS, block_threads=256),
+    dict(flags=sssp.SSSP_FLAG_WIDE_ROWS, split_degree=3),
 ]
 
 
@@ -269,7 +272,8 @@ FUZZ = [dict(), dict(grid_ctas=3), dict(block_threads=128), dict(block_threads=5
         dict(flags=sssp.SSSP_FLAG_NO_LOCAL), dict(local_max=1), dict(split_degree=1), dict(split_degree=3, grid_ctas=3),
         dict(delta_mode=1, delta_init=1), dict(delta_mode=1, delta_init=1 << 30), dict(flags=sssp.SSSP_FLAG_ADAPT_ACTIVE),
         dict(settle_head_switches=1, util_lo_pct=1000, util_hi_pct=2000), dict(flags=sssp.SSSP_FLAG_TRACE),
-        dict(flags=sssp.SSSP_FLAG_WARP_LOCAL, local_max=1, grid_ctas=2), dict(concurrent_sources=1)]
+        dict(flags=sssp.SSSP_FLAG_WARP_LOCAL, local_max=1, grid_ctas=2), dict(concurrent_sources=1),
+        dict(flags=sssp.SSSP_FLAG_WIDE_ROWS)]
 
 
 @pytest.mark.parametrize("opt", FUZZ, ids=lambda o: ",".join(f"{k}={v}" for k, v in o.items()) or "default")
@@ -437,7 +441,7 @@ def test_full_size_config(config):
     G = sssp.Graph.from_csr(g)
     H = sssp.Graph.from_csr(g, flags=sssp.SSSP_FLAG_NO_RELABEL if config == "rmat" else sssp.SSSP_FLAG_RELABEL)
     assert G.info()["relabeled"] != H.info()["relabeled"]
-    for X, opt in ((G, dict()), (G, dict(dist_bits=64)), (H, dict())):
+    for X, opt in ((G, dict()), (G, dict(flags=sssp.SSSP_FLAG_WIDE_ROWS)), (G, dict(flags=0, dist_bits=64)), (H, dict())):
         if opt:
             X.set_options(**opt)
         out = X.run(s)
