@@ -57,6 +57,7 @@ METRIC = "GTEPS (E_dij per second) and ms/source; config 5 multi-source batch on
 L2_BYTES = 126 * 2**20
 GATHER_PEAK_G = 280.0  # measured random L2 gather rate (tools/gather_bench.cu, this pool's B200)
 BATCH_K = 512
+E2E_CHUNK = 16  # sources per host-output sssp_run_batch call of the e2e pass (16 x 134 MB pinned)
 
 
 def peaks():
@@ -380,17 +381,22 @@ def run_ours(args, world, rank, local):
     units = int(tot["runs"])
     value = tot["reach_edges"] / (T / 1e3) / 1e9
 
-    # e2e through the public C ABI with host buffers: per source, the source id goes in and
-    # its full distance vector comes back to pinned host memory inside the call
+    # e2e through the public C ABI with host buffers: the sources go in and every full distance
+    # vector comes back to pinned host memory inside the call (sssp_run_batch on chunks of
+    # E2E_CHUNK sources into one pinned host buffer; the library overlaps each row's copy with
+    # the next sources' compute)
     e2e = None
     if args.e2e_steps > 0:
-        dist_h = torch.empty(g.n, dtype=torch.int64).pin_memory()
         e2e_src = mine if cfg == "batch" else mine[: args.e2e_steps]
+        chunk = max(1, min(args.e2e_chunk, len(e2e_src)))
+        dist_h = torch.empty((chunk, g.n), dtype=torch.int64).pin_memory()
         barrier(None, dev)
         t0 = time.perf_counter()
         Ee = 0
-        for s in e2e_src:
-            sssp._check(sssp.lib().sssp_run(G._h, int(s), dist_h.data_ptr(), sssp._stream_ptr(stream)))
+        for c0 in range(0, len(e2e_src), chunk):
+            part = np.ascontiguousarray(e2e_src[c0:c0 + chunk], dtype=np.uint32)
+            sssp._check(sssp.lib().sssp_run_batch(G._h, part.ctypes.data, len(part), dist_h.data_ptr(),
+                                                  sssp._stream_ptr(stream)))
             Ee += G.stats()["reach_edges"]
         torch.cuda.synchronize(dev)
         te = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
@@ -400,8 +406,9 @@ def run_ours(args, world, rank, local):
             dist.all_reduce(ee, op=dist.ReduceOp.SUM)
         e2e = {"value": ee.item() / te.item() / 1e9, "unit": "GTEPS", "h2d_bytes_per_step": 4 * len(e2e_src),
                "d2h_bytes_per_step": int(8 * g.n * len(e2e_src)), "steps": 1,
-               "path": "graph resident; sssp_run(source, pinned host dist_out) for every source of the rank's "
-                       "slice: one pass, distances copied to the host inside the call"}
+               "path": f"graph resident; sssp_run_batch(chunks of {chunk} sources, pinned host dist_out) over the "
+                       "rank's slice: one pass, every distance vector copied to the host inside the call "
+                       "(per-slot device staging rows, copies overlapped with the next sources)"}
         del dist_h
     del D
     torch.cuda.empty_cache()
@@ -462,6 +469,7 @@ def main():
     ap.add_argument("--config", default="batch", choices=list(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3, help="0 = skip the host-buffer e2e pass")
+    ap.add_argument("--e2e-chunk", type=int, default=E2E_CHUNK, help="sources per host-output batch call (e2e)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-singles", action="store_true", help="skip the single-source configs 2-4 (N=1 only)")
     ap.add_argument("--single-steps", type=int, default=5)

@@ -281,6 +281,10 @@ sssp_status sssp_run(sssp_graph *g, uint32_t source, uint64_t *dist_out, sssp_st
  * Equivalent to k calls of sssp_run (bit-identical); with
  * options.concurrent_sources = c > 1 up to c sources run concurrently (each
  * with its own workspace and stream, joined back to `stream` before return).
+ * A host dist_out (pinned for full PCIe speed) is filled through two device
+ * staging rows per slot (2*c*n*8 bytes, kept by the handle): each finished
+ * row is copied on an internal copy stream while the next sources compute,
+ * and every row is on the host when the call returns.
  * Stats cover the whole batch (batch_ms = device time of the call).  Errors as sssp_run plus
  * INVALID_ARGUMENT for k == 0 or any source >= n (checked before any work). */
 sssp_status sssp_run_batch(sssp_graph *g, const uint32_t *sources, uint32_t k,

@@ -17,6 +17,14 @@ __global__ void validate_csr_kernel(const unsigned long long* __restrict__ off, 
         if (col[e] >= n) atomicMin(&bad[1], e);
 }
 
+// A run's status block to mapped pinned host memory: posted PCIe writes, not a copy-engine job, so
+// the host's wait for a finished run never queues behind a large device->host copy in flight
+// (the host-output batch overlaps those with the next sources, sssp_lib.cu run_concurrent).
+__global__ void status_copy_kernel(const unsigned long long* __restrict__ src, unsigned long long* dst, unsigned words) {
+    for (unsigned i = threadIdx.x; i < words; i += blockDim.x) ((volatile unsigned long long*)dst)[i] = __ldcg(src + i);
+    __threadfence_system();
+}
+
 // Per-vertex row records {row begin, degree} in 32 bits for graphs with m < 2^32: the
 // throughput kernel's pop reads one aligned 8-byte record instead of two 8-byte offsets.
 __global__ void rows32_kernel(const unsigned long long* __restrict__ off, unsigned n, uint2* __restrict__ rows) {

@@ -85,9 +85,13 @@ struct Workspace {
     unsigned long long cap = 0;
     int ring_item_bytes = 0;
     unsigned trace_alloc = 0;
-    Ctl* h_ctl = nullptr;  // pinned status block
+    Ctl* h_ctl = nullptr;  // pinned status block (mapped: written by status_copy_kernel)
+    Ctl* h_ctl_dev = nullptr;  // its device alias
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
     cudaStream_t own_stream = nullptr;  // slots > 0
+    // host dist_out batches: two device staging rows per slot and the events of their host copies
+    DevBuf stage[2];
+    cudaEvent_t cev[2] = {nullptr, nullptr};
     DevBuf nf_piles, nf_cnt;            // Near-Far ablation: 4 pile buffers + counters
     unsigned long long nf_cap = 0;
     int nf_item_bytes = 0;
@@ -113,6 +117,11 @@ struct Workspace {
             if (e) cudaEventDestroy(e);
         if (own_stream) cudaStreamDestroy(own_stream);
         own_stream = nullptr;
+        for (int b = 0; b < 2; ++b) {
+            stage[b].release();
+            if (cev[b]) cudaEventDestroy(cev[b]);
+            cev[b] = nullptr;
+        }
     }
 };
 
@@ -138,6 +147,7 @@ struct sssp_graph {
     int sm_count = 0;
     std::vector<Workspace*> ws;
     DevBuf scratch, hostout, cert;
+    cudaStream_t copy_stream = nullptr;  // device -> host copies of a host-output batch
     cudaEvent_t bev[2] = {nullptr, nullptr};  // batch start / end on the caller's stream
     int cur_bits = 32;       // 64 after a 32-bit overflow was observed (sticky)
     unsigned filt_shift_hint = 0;  // 1 + filter resolution fitted to the last run's max distance
@@ -328,7 +338,8 @@ sssp_status alloc_workspace(sssp_graph* g, Workspace& w, bool own_stream) {
     CK(cudaMemset(w.bk.p, 0, sizeof(BucketCtl) * (kMaxBuckets + 1)), "bucket counters");
     CK(cudaMalloc(&w.ctl.p, sizeof(Ctl)), "allocating control block");
     CK(cudaMemset(w.ctl.p, 0, sizeof(Ctl)), "control block");
-    CK(cudaHostAlloc((void**)&w.h_ctl, sizeof(Ctl), cudaHostAllocDefault), "allocating pinned status block");
+    CK(cudaHostAlloc((void**)&w.h_ctl, sizeof(Ctl), cudaHostAllocMapped), "allocating pinned status block");
+    CK(cudaHostGetDevicePointer((void**)&w.h_ctl_dev, w.h_ctl, 0), "mapping the status block");
     std::memset(w.h_ctl, 0, sizeof(Ctl));
     for (auto& e : w.ev) CK(cudaEventCreate(&e), "creating events");
     if (own_stream) CK(cudaStreamCreateWithFlags(&w.own_stream, cudaStreamNonBlocking), "creating a slot stream");
@@ -534,7 +545,9 @@ sssp_status launch_one(sssp_graph* g, Workspace& w, uint32_t source, void* out_d
                                                         g->d_perm);
     CK(cudaGetLastError(), "finalize kernel launch");
     CK(cudaEventRecord(w.ev[3], s), "event");
-    CK(cudaMemcpyAsync(w.h_ctl, w.ctl.p, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "status copy");
+    status_copy_kernel<<<1, 256, 0, s>>>((const unsigned long long*)w.ctl.p, (unsigned long long*)w.h_ctl_dev,
+                                         (unsigned)(sizeof(Ctl) / 8));
+    CK(cudaGetLastError(), "status copy");
     w.last_grid = grid;
     w.last_block = bt;
     w.last_worker = SSSP_WORKER_CTA;
@@ -593,7 +606,9 @@ sssp_status launch_nf(sssp_graph* g, Workspace& w, uint32_t source, void* out_de
     finalize_kernel<DistT><<<aux_grid, 256, 0, s>>>(p.dist, out_dev, g->n, g->d_off, p.ctl, g->d_perm);
     CK(cudaGetLastError(), "finalize kernel launch");
     CK(cudaEventRecord(w.ev[3], s), "event");
-    CK(cudaMemcpyAsync(w.h_ctl, w.ctl.p, sizeof(Ctl), cudaMemcpyDeviceToHost, s), "status copy");
+    status_copy_kernel<<<1, 256, 0, s>>>((const unsigned long long*)w.ctl.p, (unsigned long long*)w.h_ctl_dev,
+                                         (unsigned)(sizeof(Ctl) / 8));
+    CK(cudaGetLastError(), "status copy");
     w.last_grid = grid;
     w.last_block = 256;
     w.last_worker = 0;
@@ -746,19 +761,41 @@ sssp_status classify_out(sssp_graph* g, const void* ptr, bool* is_dev) {
 
 // Concurrent batch (device dist_out): groups of c sources, one per workspace
 // and stream; every attempt of a group is launched before any is awaited.
+// c sources in flight, one per workspace slot.  Host dist_out (`host`): each slot finalizes into
+// one of its two device staging rows and the row goes to the host on the graph's copy stream
+// while the next sources compute (the copy of group i overlaps groups i+1 and i+2; a staging row
+// is rewritten only after its copy's event).
 sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, char* out, size_t esz,
-                           cudaStream_t caller, unsigned c) {
+                           cudaStream_t caller, unsigned c, bool host = false) {
     sssp_status st = ensure_slots(g, c);
     if (st) return st;
+    if (host) {
+        if (!g->copy_stream) CK(cudaStreamCreateWithFlags(&g->copy_stream, cudaStreamNonBlocking), "copy stream");
+        for (unsigned j = 0; j < c; ++j)
+            for (int b = 0; b < 2; ++b) {
+                Workspace& w = *g->ws[j];
+                if (!w.stage[b].p) {
+                    CK(cudaMalloc(&w.stage[b].p, (size_t)g->n * 8), "allocating a staging row");
+                    w.stage[b].bytes = (size_t)g->n * 8;
+                }
+                if (!w.cev[b]) CK(cudaEventCreateWithFlags(&w.cev[b], cudaEventDisableTiming), "event");
+                CK(cudaEventRecord(w.cev[b], g->copy_stream), "event");
+            }
+    }
     CK(cudaEventRecord(g->bev[0], caller), "event");
     for (unsigned j = 1; j < c; ++j) CK(cudaStreamWaitEvent(g->ws[j]->own_stream, g->bev[0], 0), "stream join");
     auto slot_stream = [&](unsigned j) { return j == 0 ? caller : g->ws[j]->own_stream; };
-    for (uint32_t i0 = 0; i0 < k && st == SSSP_OK; i0 += c) {
+    unsigned par = 0;  // staging row of this group (host output)
+    auto out_of = [&](unsigned j, uint32_t i) -> void* {
+        return host ? g->ws[j]->stage[par].p : (void*)(out + (size_t)i * g->n * esz);
+    };
+    for (uint32_t i0 = 0; i0 < k && st == SSSP_OK; i0 += c, par ^= 1u) {
         const unsigned cnt = std::min<uint32_t>(c, k - i0);
         int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
+        if (host)  // the staging row's previous copy (two groups back) has left it
+            for (unsigned j = 0; j < cnt; ++j) CK(cudaStreamWaitEvent(slot_stream(j), g->ws[j]->cev[par], 0), "stream wait");
         for (unsigned j = 0; j < cnt && st == SSSP_OK; ++j)
-            st = launch_attempt(g, *g->ws[j], sources[i0 + j], out + (size_t)(i0 + j) * g->n * esz, slot_stream(j),
-                                bits, c);
+            st = launch_attempt(g, *g->ws[j], sources[i0 + j], out_of(j, i0 + j), slot_stream(j), bits, c);
         for (unsigned j = 0; j < cnt && st == SSSP_OK; ++j) {
             const cudaError_t e = cudaStreamSynchronize(slot_stream(j));
             if (e != cudaSuccess) {
@@ -769,13 +806,22 @@ sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, c
             bool done = false;
             st = settle_attempt(g, *g->ws[j], slot_stream(j), b, 0, &done);
             if (st == SSSP_OK && !done)  // recoverable: redo this source alone (still concurrent-sized grid)
-                st = run_one_sync(g, *g->ws[j], sources[i0 + j], out + (size_t)(i0 + j) * g->n * esz, slot_stream(j),
-                                  c);
+                st = run_one_sync(g, *g->ws[j], sources[i0 + j], out_of(j, i0 + j), slot_stream(j), c);
+            if (st == SSSP_OK && host) {  // the row is final (slot stream synchronized): send it home
+                cudaError_t e = cudaMemcpyAsync(out + (size_t)(i0 + j) * g->n * esz, g->ws[j]->stage[par].p,
+                                                (size_t)g->n * esz, cudaMemcpyDeviceToHost, g->copy_stream);
+                if (e == cudaSuccess) e = cudaEventRecord(g->ws[j]->cev[par], g->copy_stream);
+                if (e != cudaSuccess) st = cuda_fail(e, "copying dist to host");
+            }
         }
     }
     for (unsigned j = 1; j < c; ++j) {
         cudaEventRecord(g->ws[j]->ev[3], g->ws[j]->own_stream);
         cudaStreamWaitEvent(caller, g->ws[j]->ev[3], 0);
+    }
+    if (host) {
+        const cudaError_t e = cudaStreamSynchronize(g->copy_stream);  // host rows complete on return
+        if (e != cudaSuccess && st == SSSP_OK) st = cuda_fail(e, "copying dist to host");
     }
     return st;
 }
@@ -808,7 +854,7 @@ sssp_status run_many(sssp_graph* g, const uint32_t* sources, uint32_t k, void* d
     const unsigned c = g->opts.algorithm == SSSP_ALGO_NEAR_FAR
                            ? 1u  // grid-wide barriers: one cooperative launch at a time
                            : std::min<unsigned>(std::max(1u, g->opts.concurrent_sources), k);
-    g->stats.concurrency = (is_dev && c > 1) ? c : 1;
+    g->stats.concurrency = c > 1 ? c : 1;
     const bool async = (g->opts.flags & SSSP_FLAG_ASYNC) && is_dev && k == 1;
     if (!is_dev && !g->hostout.p) {
         cudaError_t e = cudaMalloc(&g->hostout.p, (size_t)g->n * 8);
@@ -819,8 +865,8 @@ sssp_status run_many(sssp_graph* g, const uint32_t* sources, uint32_t k, void* d
         g->hostout.bytes = (size_t)g->n * 8;
     }
     cudaEventRecord(g->bev[0], s);
-    if (is_dev && c > 1) {
-        st = run_concurrent(g, sources, k, (char*)dist_out, esz, s, c);
+    if (c > 1) {  // (host dist_out: staged per slot, copies overlapped with the next sources)
+        st = run_concurrent(g, sources, k, (char*)dist_out, esz, s, c, !is_dev);
     } else {
         for (uint32_t i = 0; i < k && st == SSSP_OK; ++i) {
             void* out = is_dev ? (void*)((char*)dist_out + (size_t)i * g->n * esz) : g->hostout.p;
@@ -1126,6 +1172,7 @@ sssp_status sssp_graph_destroy(sssp_graph* g) {
     if (!g) return SSSP_OK;
     DeviceGuard dg(g->device);
     cudaDeviceSynchronize();
+    if (g->copy_stream) cudaStreamDestroy(g->copy_stream);
     if (g->d_off) cudaFree(g->d_off);
     if (g->d_adj) cudaFree(g->d_adj);
     if (g->d_rows) cudaFree(g->d_rows);

@@ -528,6 +528,34 @@ def test_concurrent_batch(conc):
         assert np.array_equal(sssp.to_u64(D[i]), oracle.dijkstra(g, int(s))[0])
 
 
+@pytest.mark.parametrize("conc,pinned", [(1, True), (2, True), (3, False)])
+def test_batch_host_out(conc, pinned):
+    """Host dist_out batches: staged per slot, copies overlapped with the next sources."""
+    import torch
+    g = gg.make("rmat", scale_down=8)
+    srcs = gg.config_sources("rmat", g, 5)
+    G = sssp.Graph.from_csr(g, concurrent_sources=conc)
+    out = torch.full((len(srcs), g.n), -7, dtype=torch.int64)
+    if pinned:
+        out = out.pin_memory()
+    G.run_batch(srcs, out=out)
+    assert G.stats()["concurrency"] == conc
+    for i, s in enumerate(srcs):
+        assert np.array_equal(sssp.to_u64(out[i]), oracle.dijkstra(g, int(s))[0])
+
+
+def test_batch_host_out_overflow_retry():
+    import torch
+    g = gg.make("road", scale_down=8)
+    srcs = gg.config_sources("road", g, 5)
+    G = sssp.Graph.from_csr(g, concurrent_sources=2, ring_items=64)
+    out = torch.empty((len(srcs), g.n), dtype=torch.int64)
+    G.run_batch(srcs, out=out)
+    assert G.stats()["retries"] >= 1
+    for i, s in enumerate(srcs):
+        assert np.array_equal(sssp.to_u64(out[i]), oracle.dijkstra(g, int(s))[0])
+
+
 def test_concurrent_batch_with_overflow_retry():
     g = gg.make("road", scale_down=8)
     srcs = gg.config_sources("road", g, 4)
