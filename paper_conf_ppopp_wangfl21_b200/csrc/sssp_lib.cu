@@ -12,6 +12,8 @@
 #include <string>
 #include <type_traits>
 #include <vector>
+#include <thread>
+#include <chrono>
 
 #include "../../include/sssp.h"
 #include "adds_kernel.cuh"
@@ -785,36 +787,62 @@ sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, c
     CK(cudaEventRecord(g->bev[0], caller), "event");
     for (unsigned j = 1; j < c; ++j) CK(cudaStreamWaitEvent(g->ws[j]->own_stream, g->bev[0], 0), "stream join");
     auto slot_stream = [&](unsigned j) { return j == 0 ? caller : g->ws[j]->own_stream; };
-    unsigned par = 0;  // staging row of this group (host output)
+    // Every slot runs its own sequence: when a slot's source finishes (stream query), it is
+    // settled and the slot starts the next source at once -- no slot waits for the slowest
+    // source of a group.
+    constexpr uint32_t kNone = 0xFFFFFFFFu;
+    std::vector<uint32_t> run_i(c, kNone);  // source index running in slot j
+    std::vector<int> run_bits(c, 32);
+    std::vector<unsigned> spar(c, 1u);      // slot j's staging row (host output)
+    uint32_t next = 0;
+    unsigned active = 0;
     auto out_of = [&](unsigned j, uint32_t i) -> void* {
-        return host ? g->ws[j]->stage[par].p : (void*)(out + (size_t)i * g->n * esz);
+        return host ? g->ws[j]->stage[spar[j]].p : (void*)(out + (size_t)i * g->n * esz);
     };
-    for (uint32_t i0 = 0; i0 < k && st == SSSP_OK; i0 += c, par ^= 1u) {
-        const unsigned cnt = std::min<uint32_t>(c, k - i0);
-        int bits = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
-        if (host)  // the staging row's previous copy (two groups back) has left it
-            for (unsigned j = 0; j < cnt; ++j) CK(cudaStreamWaitEvent(slot_stream(j), g->ws[j]->cev[par], 0), "stream wait");
-        for (unsigned j = 0; j < cnt && st == SSSP_OK; ++j)
-            st = launch_attempt(g, *g->ws[j], sources[i0 + j], out_of(j, i0 + j), slot_stream(j), bits, c);
-        for (unsigned j = 0; j < cnt && st == SSSP_OK; ++j) {
-            const cudaError_t e = cudaStreamSynchronize(slot_stream(j));
-            if (e != cudaSuccess) {
-                st = cuda_fail(e, "SSSP run");
+    auto start = [&](unsigned j) -> sssp_status {
+        const uint32_t i = next++;
+        if (host) {  // the staging row's previous copy (two sources back on this slot) has left it
+            spar[j] ^= 1u;
+            CK(cudaStreamWaitEvent(slot_stream(j), g->ws[j]->cev[spar[j]], 0), "stream wait");
+        }
+        run_i[j] = i;
+        run_bits[j] = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
+        ++active;
+        return launch_attempt(g, *g->ws[j], sources[i], out_of(j, i), slot_stream(j), run_bits[j], c);
+    };
+    for (unsigned j = 0; j < c && next < k && st == SSSP_OK; ++j) st = start(j);
+    while (active && st == SSSP_OK) {
+        bool any = false;
+        for (unsigned j = 0; j < c && st == SSSP_OK; ++j) {
+            if (run_i[j] == kNone) continue;
+            const cudaError_t q = cudaStreamQuery(slot_stream(j));
+            if (q == cudaErrorNotReady) continue;
+            if (q != cudaSuccess) {
+                st = cuda_fail(q, "SSSP run");
                 break;
             }
-            int b = bits;
+            any = true;
+            const uint32_t i = run_i[j];
+            int b = run_bits[j];
             bool done = false;
             st = settle_attempt(g, *g->ws[j], slot_stream(j), b, 0, &done);
             if (st == SSSP_OK && !done)  // recoverable: redo this source alone (still concurrent-sized grid)
-                st = run_one_sync(g, *g->ws[j], sources[i0 + j], out_of(j, i0 + j), slot_stream(j), c);
-            if (st == SSSP_OK && host) {  // the row is final (slot stream synchronized): send it home
-                cudaError_t e = cudaMemcpyAsync(out + (size_t)(i0 + j) * g->n * esz, g->ws[j]->stage[par].p,
+                st = run_one_sync(g, *g->ws[j], sources[i], out_of(j, i), slot_stream(j), c);
+            if (st == SSSP_OK && host) {  // the row is final: send it home on the copy stream
+                cudaError_t e = cudaMemcpyAsync(out + (size_t)i * g->n * esz, g->ws[j]->stage[spar[j]].p,
                                                 (size_t)g->n * esz, cudaMemcpyDeviceToHost, g->copy_stream);
-                if (e == cudaSuccess) e = cudaEventRecord(g->ws[j]->cev[par], g->copy_stream);
+                if (e == cudaSuccess) e = cudaEventRecord(g->ws[j]->cev[spar[j]], g->copy_stream);
                 if (e != cudaSuccess) st = cuda_fail(e, "copying dist to host");
             }
+            run_i[j] = kNone;
+            --active;
+            if (st == SSSP_OK && next < k) st = start(j);
         }
+        if (!any && st == SSSP_OK) std::this_thread::sleep_for(std::chrono::microseconds(5));
     }
+    if (st != SSSP_OK)  // drain the slots still running before the workspaces are reused
+        for (unsigned j = 0; j < c; ++j)
+            if (run_i[j] != kNone) cudaStreamSynchronize(slot_stream(j));
     for (unsigned j = 1; j < c; ++j) {
         cudaEventRecord(g->ws[j]->ev[3], g->ws[j]->own_stream);
         cudaStreamWaitEvent(caller, g->ws[j]->ev[3], 0);
