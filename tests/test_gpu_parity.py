@@ -556,6 +556,22 @@ def test_batch_host_out_overflow_retry():
         assert np.array_equal(sssp.to_u64(out[i]), oracle.dijkstra(g, int(s))[0])
 
 
+@pytest.mark.parametrize("host", [False, True])
+def test_independent_slots_ragged_with_retries(host):
+    """7 sources on 3 slots (a ragged last round), every source overflowing its 64-item ring
+    first: slots settle, retry and restart out of step with each other."""
+    import torch
+    g = gg.make("rmat", scale_down=9)
+    srcs = gg.config_sources("rmat", g, 7)
+    G = sssp.Graph.from_csr(g, concurrent_sources=3, ring_items=64)
+    out = torch.empty((len(srcs), g.n), dtype=torch.int64) if host else None
+    D = G.run_batch(srcs, out=out)
+    st = G.stats()
+    assert st["retries"] >= 1 and st["concurrency"] == 3
+    for i, s in enumerate(srcs):
+        assert np.array_equal(sssp.to_u64(D[i]), oracle.dijkstra(g, int(s))[0])
+
+
 def test_concurrent_batch_with_overflow_retry():
     g = gg.make("road", scale_down=8)
     srcs = gg.config_sources("road", g, 4)
