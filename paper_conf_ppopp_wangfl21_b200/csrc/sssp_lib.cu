@@ -794,6 +794,7 @@ sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, c
     std::vector<uint32_t> run_i(c, kNone);  // source index running in slot j
     std::vector<int> run_bits(c, 32);
     std::vector<unsigned> spar(c, 1u);      // slot j's staging row (host output)
+    std::vector<int> tries(c, 0);           // attempts of the running source (overflow re-runs)
     uint32_t next = 0;
     unsigned active = 0;
     auto out_of = [&](unsigned j, uint32_t i) -> void* {
@@ -807,6 +808,7 @@ sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, c
         }
         run_i[j] = i;
         run_bits[j] = g->opts.dist_bits ? (int)g->opts.dist_bits : g->cur_bits;
+        tries[j] = 0;
         ++active;
         return launch_attempt(g, *g->ws[j], sources[i], out_of(j, i), slot_stream(j), run_bits[j], c);
     };
@@ -825,9 +827,13 @@ sssp_status run_concurrent(sssp_graph* g, const uint32_t* sources, uint32_t k, c
             const uint32_t i = run_i[j];
             int b = run_bits[j];
             bool done = false;
-            st = settle_attempt(g, *g->ws[j], slot_stream(j), b, 0, &done);
-            if (st == SSSP_OK && !done)  // recoverable: redo this source alone (still concurrent-sized grid)
-                st = run_one_sync(g, *g->ws[j], sources[i], out_of(j, i), slot_stream(j), c);
+            st = settle_attempt(g, *g->ws[j], slot_stream(j), b, tries[j], &done);
+            if (st == SSSP_OK && !done) {  // recoverable (ring regrown / 64-bit): re-run it on this slot,
+                run_bits[j] = b;             // without holding up the other slots
+                if (++tries[j] >= 24) st = fail(SSSP_ERR_WORKLIST_OVERFLOW, "retries exhausted");
+                else st = launch_attempt(g, *g->ws[j], sources[i], out_of(j, i), slot_stream(j), b, c);
+                continue;
+            }
             if (st == SSSP_OK && host) {  // the row is final: send it home on the copy stream
                 cudaError_t e = cudaMemcpyAsync(out + (size_t)i * g->n * esz, g->ws[j]->stage[spar[j]].p,
                                                 (size_t)g->n * esz, cudaMemcpyDeviceToHost, g->copy_stream);
