@@ -260,7 +260,11 @@ bool chunked_ring(const sssp_graph* g) { return (g->opts.flags & SSSP_FLAG_CHUNK
 unsigned long long default_cap(const sssp_graph* g) {
     if (g->opts.ring_items) return next_pow2(std::max<unsigned long long>(g->opts.ring_items, 64ull));
     if (chunked_ring(g)) return next_pow2(std::max<unsigned long long>(2ull * g->n, 1ull << 18));
-    return next_pow2(std::max<unsigned long long>((unsigned long long)g->n, 1ull << 16));
+    // road-like graphs (the latency build): 2n per slot -- at n = 2^24 ROAD overflowed 2^24-item
+    // slots on some sources (the clip slot collects most of a run's far pushes), and each overflow
+    // costs a full re-run (bench singles 31 -> 45 ms/source with two of them)
+    const unsigned long long base = warp_local_on(g) ? 2ull * g->n : (unsigned long long)g->n;
+    return next_pow2(std::max<unsigned long long>(base, 1ull << 16));
 }
 
 sssp_status ensure_ring(sssp_graph* g, Workspace& w, int item_bytes, unsigned long long cap) {
