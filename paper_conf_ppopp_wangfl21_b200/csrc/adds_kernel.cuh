@@ -119,7 +119,7 @@ __device__ __forceinline__ long long warp_sum_s64(long long x) {
 // steps) since the last Delta change; a change needs since >= settle (a quarter
 // of that for growth while the re-expansion share is below waste_lo / 8).
 struct CtlDecision {
-    unsigned k, A, flo, since, ceil;
+    unsigned k, A, flo, since, ceil, pk;
     bool changed;
     unsigned flags;  // decision inputs, recorded in the trace: 1 low, 2 high, 4 beyond, 8 wasteful,
                      // 16 frugal, 32 clipping, 64 waste known, 128 progressed, 256 settled
@@ -130,14 +130,15 @@ struct CtlDecision {
 // over the recent window.  clip = share of recent pushes that were clipped.
 template <typename DistT>
 __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, unsigned flo, unsigned since,
-                              unsigned ceil, bool head_switch, long long total, long long tail, long long win, unsigned waste,
+                              unsigned ceil, unsigned pk, bool head_switch, long long total, long long tail, long long win,
+                              unsigned waste,
                               bool waste_known, unsigned clip, bool clip_known, unsigned ratio_x100,
                               bool progressed, long long busy) {
     // since = [0,8) controller steps, [8,16) head switches since the last change
     unsigned steps = since & 0xffu, hsw = (since >> 8) & 0xffu;
     steps = steps < 255u ? steps + 1 : 255u;
     if (head_switch && hsw < 255u) ++hsw;
-    CtlDecision d{k, A, flo, steps | (hsw << 8), ceil, false, 0u};
+    CtlDecision d{k, A, flo, steps | (hsw << 8), ceil, head_switch ? 0u : pk, false, 0u};
     if (!p.dynamic) return d;
     // the waste ceiling (hysteresis, below) holds for the rest of the run: letting it expire
     // after 64 or 16 head switches regrew ROAD into wasteful Deltas (work 1.63x -> 2.0x,
@@ -181,12 +182,15 @@ __device__ CtlDecision decide(const Params<DistT>& p, unsigned k, unsigned A, un
         d.flo = d.k;
         if (d.ceil <= d.k) d.ceil = 0xffu;  // the clip bound overrides the waste ceiling
         d.changed = true;
-    } else if (wasteful && k > flo && steps >= 4 * p.settle && hsw == 0) {
+    } else if (wasteful && k > flo && steps >= 4 * p.settle && hsw == 0 && d.pk < 2u) {
         // sustained waste while the head does not move (one bucket holding the whole frontier:
         // RMAT with U[1,2^20] re-expanded 6x at 2^15 with the head parked for 20 ms): shrink
-        // after four settling periods even without head switches
+        // after four settling periods even without head switches -- at most twice before the
+        // head moves again (a correction wave runs on whatever Delta: ROAD collapsed 2^11 -> 2^2
+        // this way, every step reading 100 % re-expansions, and then crawled; r02 §12)
         d.k = k - 1;
         d.ceil = k;
+        d.pk = d.pk + 1u;
         d.changed = true;
     } else if (steps >= p.settle && turned) {
         if (wasteful && k > flo) {
@@ -339,13 +343,14 @@ __device__ bool try_advance(const Params<DistT>& p, const Head hd, const int lan
     bool known, cknown;
     const unsigned waste = recent_waste(p, known);
     const unsigned clip = recent_clip(p, cknown);
-    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), meta_ceil(hd.meta), true, total, tail, win, waste,
+    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), meta_ceil(hd.meta), meta_pk(hd.meta), true,
+                                 total, tail, win, waste,
                                  known, clip, cknown, cumulative_ratio(p),
                                  ld_relaxed_u64(&p.ctl->g_exp) >= p.startup_first ||
                                      ld_relaxed_u32(&p.ctl->head_switches) >= 32u,
                                  (long long)ld_relaxed_u64(&p.ctl->g_busy));
     const Head nhd{rehead(hd.h + o, k, d.k),
-                   pack_meta((hs + o) & (nb - 1), d.k, d.A, d.flo, d.since, d.ceil)};
+                   pack_meta((hs + o) & (nb - 1), d.k, d.A, d.flo, d.since, d.ceil, d.pk)};
     SSSP_FUZZ_AT(FZ_HEAD);
     commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 1u, d.flags, clip, cknown);
     return false;
@@ -366,12 +371,13 @@ __device__ void periodic_step(const Params<DistT>& p, const int lane) {
     bool known, cknown;
     const unsigned waste = recent_waste(p, known);
     const unsigned clip = recent_clip(p, cknown);
-    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), meta_ceil(hd.meta), false, total, tail, win, waste,
+    const CtlDecision d = decide(p, k, A, meta_floor(hd.meta), meta_since(hd.meta), meta_ceil(hd.meta), meta_pk(hd.meta), false,
+                                 total, tail, win, waste,
                                  known, clip, cknown, cumulative_ratio(p),
                                  ld_relaxed_u64(&p.ctl->g_exp) >= p.startup_first ||
                                      ld_relaxed_u32(&p.ctl->head_switches) >= 32u,
                                  (long long)ld_relaxed_u64(&p.ctl->g_busy));
-    const Head nhd{rehead(hd.h, k, d.k), pack_meta(hs, d.k, d.A, d.flo, d.since, d.ceil)};
+    const Head nhd{rehead(hd.h, k, d.k), pack_meta(hs, d.k, d.A, d.flo, d.since, d.ceil, d.pk)};
     commit_step(p, hd, nhd, d.k != k, d.since, total, win, tail, waste, 2u, d.flags, clip, cknown);
 }
 

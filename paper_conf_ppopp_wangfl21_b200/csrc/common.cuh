@@ -97,10 +97,12 @@ struct alignas(16) Head {
 };
 
 __host__ __device__ __forceinline__ unsigned long long pack_meta(unsigned hs, unsigned k, unsigned A,
-                                                                 unsigned flo, unsigned since, unsigned ceil = 0xffu) {
+                                                                 unsigned flo, unsigned since, unsigned ceil = 0xffu,
+                                                                 unsigned pk = 0u) {
     return (unsigned long long)(hs & 0xff) | ((unsigned long long)(k & 0xff) << 8) |
            ((unsigned long long)(A & 0xff) << 16) | ((unsigned long long)(flo & 0xff) << 24) |
-           ((unsigned long long)(since & 0xffff) << 32) | ((unsigned long long)(ceil & 0xff) << 48);
+           ((unsigned long long)(since & 0xffff) << 32) | ((unsigned long long)(ceil & 0xff) << 48) |
+           ((unsigned long long)(pk & 0xff) << 56);
 }
 __host__ __device__ __forceinline__ unsigned meta_hs(unsigned long long m) { return (unsigned)(m & 0xff); }
 __host__ __device__ __forceinline__ unsigned meta_k(unsigned long long m) { return (unsigned)((m >> 8) & 0xff); }
@@ -108,6 +110,8 @@ __host__ __device__ __forceinline__ unsigned meta_A(unsigned long long m) { retu
 __host__ __device__ __forceinline__ unsigned meta_floor(unsigned long long m) { return (unsigned)((m >> 24) & 0xff); }
 __host__ __device__ __forceinline__ unsigned meta_since(unsigned long long m) { return (unsigned)((m >> 32) & 0xffff); }
 __host__ __device__ __forceinline__ unsigned meta_ceil(unsigned long long m) { return (unsigned)((m >> 48) & 0xff); }
+// [56,64) parked shrinks since the head last switched (bounds the shrink-without-head-switch rule)
+__host__ __device__ __forceinline__ unsigned meta_pk(unsigned long long m) { return (unsigned)((m >> 56) & 0xff); }
 
 struct TraceEntry {  // mirrors sssp_trace_entry
     unsigned long long time_ns, head, pending_total, pending_window, pending_tail;
