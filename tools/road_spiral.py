@@ -15,9 +15,10 @@ import paper_conf_ppopp_wangfl21_b200 as sssp  # noqa: E402
 def main():
     cfg = sys.argv[1] if len(sys.argv) > 1 else "road"
     reps = int(sys.argv[2]) if len(sys.argv) > 2 else 3
+    trace = "notrace" not in sys.argv
     g = gg.make(cfg)
     srcs = gg.config_sources(cfg, g, 8)
-    G = sssp.Graph.from_csr(g, flags=sssp.SSSP_FLAG_TRACE)
+    G = sssp.Graph.from_csr(g, flags=sssp.SSSP_FLAG_TRACE if trace else 0)
     worst = None
     for r in range(reps):
         for s in srcs:
@@ -28,8 +29,10 @@ def main():
                               "k0": st["init_delta_log2"], "k": st["final_delta_log2"],
                               "changes": st["delta_changes"], "switches": st["head_switches"]}), flush=True)
             if worst is None or w > worst[0]:
-                worst = (w, int(s), G.trace())
+                worst = (w, int(s), G.trace() if trace else [])
     w, s, tr = worst
+    if not tr:
+        return
     print(f"# worst run: source {s}, work {w:.3f}; Delta / A changes:")
     t0 = tr[0]["time_ns"]
     for i in range(1, len(tr)):
