@@ -57,7 +57,8 @@ METRIC = "GTEPS (E_dij per second) and ms/source; config 5 multi-source batch on
 L2_BYTES = 126 * 2**20
 GATHER_PEAK_G = 280.0  # measured random L2 gather rate (tools/gather_bench.cu, this pool's B200)
 BATCH_K = 512
-E2E_CHUNK = 16  # sources per host-output sssp_run_batch call of the e2e pass (16 x 134 MB pinned)
+E2E_CHUNK = 64  # sources per host-output sssp_run_batch call of the e2e pass (64 x 134 MB = 8.6 GB pinned):
+                # each call ends with its last copies unoverlapped (16: e2e 65.6-67.7, 64: 72.5-74.8 GTEPS)
 
 
 def peaks():
